@@ -1,0 +1,217 @@
+/*
+ * ac.h -- C ABI of the B200-native Aho-Corasick matching scan (libac.so).
+ *
+ * Paper: N.-P. Tran, M. Lee, S. Hong, J. Choi, "High Throughput Parallel
+ * Implementation of Aho-Corasick Algorithm on a GPU", IPDPS-W 2013.
+ * Citations "P:<line>" refer to the paper text line numbers.
+ *
+ * The two calls follow the paper's problem statement: "In the first
+ * phase, a pattern matching machine called AC automaton (machine) is
+ * constructed from a finite set of patterns.  In the second phase, the input
+ * text data is applied to the constructed AC machine in order to find the
+ * locations that the patterns appear."
+ *   - ac_build  : phase 1.  Host-side construction of the DFA (next-move
+ *                 function delta with the failure function folded in) as a
+ *                 State Transition Table (STT, Fig. 5), built once on
+ *                 one CPU core and copied to device memory.  Untimed,
+ *                 like the paper.
+ *   - ac_match  : phase 2.  The data-parallel scan: one STT transition per
+ *                 text byte (O(n)), every (position, pattern)
+ *                 occurrence emitted, on an sm_100a GPU.
+ *
+ * Conventions:
+ *   - Alphabet: raw bytes 0..255, binary safe, case sensitive (R7).
+ *   - Pattern ids are the 0-based indices of the input array (R4);
+ *     duplicate patterns are distinct ids (R5); empty patterns are rejected
+ *     (R6).
+ *   - Every occurrence is reported, overlapping and nested ones included
+ *     (R19).
+ *   - A match record is one 64-bit word:  (start << 24) | pattern
+ *     where start is the 0-based index of the occurrence's first byte and
+ *     end = start + len(pattern) - 1 is the paper's "end of position" (
+ *     R2).  Canonical order = ascending record value = (start, pattern)
+ *     ascending (R3).  Hence n < 2^40 and n_patterns < 2^24.
+ *   - All functions are thread safe; an ac_stt is immutable after ac_build,
+ *     so concurrent ac_match calls on different streams are allowed.
+ *   - No C++ exception or abort crosses this ABI.  Errors are status codes;
+ *     ac_last_error() returns a thread-local detail string.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default).
+ *   - There is no CPU fallback: without a usable sm_100 device every device
+ *     call returns AC_ERR_NO_DEVICE or AC_ERR_CUDA.
+ */
+#ifndef AC_H
+#define AC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef uint64_t ac_match_t;
+#define AC_MATCH_START(m) ((uint64_t)(m) >> 24)
+#define AC_MATCH_PATTERN(m) ((uint32_t)((m) & 0xFFFFFFu))
+#define AC_MAX_PATTERNS (1u << 24)
+#define AC_MAX_TEXT ((uint64_t)1 << 40)
+
+typedef enum {
+    AC_OK = 0,
+    AC_ERR_INVALID_ARG = 1,   /* NULL pointer, bad option, ...              */
+    AC_ERR_EMPTY_PATTERN = 2, /* some lens[i] == 0 (reading R6)             */
+    AC_ERR_TOO_LARGE = 3,     /* n_patterns >= 2^24, states >= 2^31, n >= 2^40 */
+    AC_ERR_CAPACITY = 4,      /* list longer than cap: *count = needed size  */
+    AC_ERR_NO_MEMORY = 5,     /* host or device allocation failed           */
+    AC_ERR_CUDA = 6,          /* any CUDA runtime/driver error              */
+    AC_ERR_NO_DEVICE = 7      /* no usable compute-capability-10.x device   */
+} ac_status;
+
+/* Opaque device STT handle: dense transition table + class map + output
+ * CSR + pattern lengths, owned by the library, released by ac_free(). */
+typedef struct ac_stt ac_stt;
+
+/* Opaque HOST table (phase-1 result before upload); used by tests to check
+ * the builder without a GPU. */
+typedef struct ac_table ac_table;
+
+/* STT residency tiers. */
+enum { AC_TIER_AUTO = 0, AC_TIER_SMEM = 1, AC_TIER_HYBRID = 2, AC_TIER_GLOBAL = 3 };
+
+typedef struct {
+    uint32_t struct_size;  /* sizeof(ac_build_opts)                          */
+    uint32_t entry_bytes;  /* 0 = auto (2 if states <= 32768 else 4), 2 or 4 */
+    uint32_t tier;         /* AC_TIER_*                                      */
+    uint32_t hot_rows;     /* HYBRID: rows kept in shared memory (0 = auto)  */
+    uint32_t forward;      /* 0 (default) = automaton of the REVERSED
+                              patterns, scanned right-to-left so that matches
+                              come out in canonical (start, pattern) order;
+                              1 = the paper's forward automaton (tests only:
+                              ac_build rejects it, ac_compile accepts it)    */
+} ac_build_opts;
+
+typedef struct {
+    uint32_t n_patterns;
+    uint32_t n_states;     /* S                                             */
+    uint32_t n_classes;    /* C: class 0 = bytes in no pattern              */
+    uint32_t row_stride;   /* entries per STT row (>= C, padded)            */
+    uint32_t entry_bytes;  /* 2 or 4                                        */
+    uint32_t tier;         /* resolved AC_TIER_*                            */
+    uint32_t hot_rows;     /* rows resident in shared memory                */
+    uint32_t maxlen;       /* longest pattern                               */
+    uint32_t forward;
+    uint32_t reserved;
+    uint64_t stt_bytes;    /* S * row_stride * entry_bytes                  */
+    uint64_t out_entries;  /* sum over states of |output(s)|                */
+} ac_stt_info;
+
+/* Scan variants (SURVEY 8(f) NEXT-1 ablations are selectable here). */
+enum {
+    AC_KERNEL_AUTO = 0,
+    AC_KERNEL_STAGED = 1, /* TMA-staged text tiles in shared memory, the
+                             B200 form of the paper's "shared memory
+                             approach"                           */
+    AC_KERNEL_GLOBAL = 2  /* text read straight from global memory, the
+                             paper's "global memory only approach" */
+};
+
+typedef struct {
+    uint32_t struct_size;  /* sizeof(ac_match_opts)                          */
+    uint32_t kernel;       /* AC_KERNEL_*                                    */
+    uint32_t chain_bytes;  /* bytes owned per thread chain (0 = auto; STAGED:
+                              rounded to the tile width)                     */
+    uint32_t n_events;     /* pairs available in `events`                    */
+    void **events;         /* optional cudaEvent_t[2 * n_events]: events[2i]
+                              and events[2i+1] are recorded on the stream
+                              right before / after kernel launch i, so a
+                              caller can time each kernel (bench.py)         */
+} ac_match_opts;
+
+/* Per-call device result written by the async entry points. */
+typedef struct {
+    uint64_t count;        /* total occurrences (always valid)               */
+    uint32_t status;       /* AC_OK or AC_ERR_CAPACITY                       */
+    uint32_t reserved;
+} ac_result;
+
+/* ---------------------------------------------------------------- phase 1
+ * ac_build: patterns[i] points to lens[i] bytes (host memory, any bytes).
+ * Builds the DFA on the host, uploads it to `device`, returns a
+ * handle in *out.  Errors: AC_ERR_INVALID_ARG (NULL args, opts->forward),
+ * AC_ERR_EMPTY_PATTERN, AC_ERR_TOO_LARGE, AC_ERR_NO_MEMORY, AC_ERR_CUDA,
+ * AC_ERR_NO_DEVICE.  `opts` may be NULL (all auto). */
+ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n_patterns,
+                   int device, const ac_build_opts *opts, ac_stt **out);
+void ac_free(ac_stt *stt);
+ac_status ac_stt_query(const ac_stt *stt, ac_stt_info *info);
+/* Copies the n_patterns pattern lengths to host memory `lens`. */
+ac_status ac_stt_pattern_lengths(const ac_stt *stt, uint32_t *lens);
+
+/* ---------------------------------------------------------------- phase 2
+ * ac_match: scans d_text[0, n) (DEVICE memory, any alignment, n may be 0)
+ * and reports every occurrence.
+ *   d_out == NULL : count only; *count = number of occurrences.
+ *   d_out != NULL : DEVICE buffer of `cap` records; on AC_OK it holds the
+ *                   *count records in canonical order.  If the count exceeds
+ *                   cap, returns AC_ERR_CAPACITY with *count = required size
+ *                   and d_out contents unspecified.
+ * The call is stream-ordered on `stream` and synchronises it before
+ * returning (it must return the count).  Scratch space is taken from the
+ * stream-ordered allocator (cudaMallocAsync). */
+ac_status ac_match(const ac_stt *stt, const uint8_t *d_text, uint64_t n, ac_match_t *d_out,
+                   uint64_t cap, uint64_t *count, void *stream);
+
+/* ac_match_shard: one shard of a larger text.  d_text[0,
+ * n_owned + n_halo) is readable; occurrences whose start lies in [0, n_owned)
+ * are reported, with start + base in the records.  The caller passes
+ * n_halo = min(maxlen - 1, n_total - (base + n_owned)) bytes of the next
+ * shard so straddling occurrences are found exactly once (R8/R9). */
+ac_status ac_match_shard(const ac_stt *stt, const uint8_t *d_text, uint64_t n_owned,
+                         uint64_t n_halo, uint64_t base, ac_match_t *d_out, uint64_t cap,
+                         uint64_t *count, void *stream);
+
+/* Asynchronous form of ac_match_shard: enqueues the whole scan on `stream`
+ * and returns without synchronising; the count and status land in the
+ * DEVICE struct *d_result when the stream reaches that point.  `opts` may be
+ * NULL.  Host-side argument errors are returned immediately. */
+ac_status ac_match_async(const ac_stt *stt, const uint8_t *d_text, uint64_t n_owned,
+                         uint64_t n_halo, uint64_t base, ac_match_t *d_out, uint64_t cap,
+                         ac_result *d_result, void *stream, const ac_match_opts *opts);
+
+/* Number of kernel launches the last ac_match_async on this thread issued,
+ * and the name of launch i (NULL if out of range). */
+uint32_t ac_last_launch_count(void);
+const char *ac_last_launch_name(uint32_t i);
+
+/* End-to-end entry with HOST buffers: copies h_text[0,n) to the device,
+ * scans it, copies the count and (if h_out != NULL) the canonical list back
+ * into h_out[0, cap).  Same status semantics as ac_match.  Device staging is
+ * allocated on `stream`'s device with the stream-ordered allocator. */
+ac_status ac_match_host(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac_match_t *h_out,
+                        uint64_t cap, uint64_t *count, void *stream);
+
+/* ----------------------------------------------------- host-only builder
+ * ac_compile: phase 1 without a device (for tests and tooling).  opts->tier
+ * and hot_rows are ignored; opts->forward selects the paper's forward
+ * automaton.  ac_table_export copies any non-NULL array out:
+ *   class_map[256]            byte -> class
+ *   stt[S * row_stride]       entries of entry_bytes each: low bits = next
+ *                             state, top bit (15 or 31) = output(next) != {}
+ *   out_off[S + 1], out_ids[out_entries]   output CSR, ids ascending
+ */
+ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n_patterns,
+                     const ac_build_opts *opts, ac_table **out);
+ac_status ac_table_query(const ac_table *t, ac_stt_info *info);
+ac_status ac_table_export(const ac_table *t, uint8_t *class_map, void *stt, uint32_t *out_off,
+                          uint32_t *out_ids);
+void ac_table_free(ac_table *t);
+
+/* ------------------------------------------------------------ diagnostics */
+const char *ac_status_string(ac_status s);
+const char *ac_last_error(void);
+/* Library build identification, e.g. "libac sm_100a". */
+const char *ac_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* AC_H */

@@ -1,0 +1,589 @@
+// ac_abi.cu -- the C ABI of libac (include/ac.h): validation, STT upload and
+// residency planning, scan planning and launch sequencing.
+//
+// Phase split follows the paper: the STT is built once on the host and
+// copied to the device; the text is device resident before the scan
+// (P:148); build and copies are outside the timed scan.
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+
+#include <cudaTypedefs.h>
+
+#include "ac_internal.h"
+#include "ac_scan.cuh"
+
+namespace acx {
+
+static thread_local std::string g_err;
+static thread_local uint32_t g_launches = 0;
+static thread_local const char *g_names[16];
+
+void set_error(const std::string &msg) { g_err = msg; }
+
+static ac_status cuda_fail(cudaError_t e, const char *what) {
+    set_error(std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")");
+    return AC_ERR_CUDA;
+}
+
+#define AC_CUDA(call, what)                          \
+    do {                                             \
+        cudaError_t e_ = (call);                     \
+        if (e_ != cudaSuccess) return cuda_fail(e_, what); \
+    } while (0)
+
+static const StagedConfig kStaged{256, 2, 64, 3};
+static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
+static const uint64_t kStagedMinBytes = 64 * 1024;
+static const uint64_t kStagedMinChain = 256;
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda).
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    });
+    return fn;
+}
+
+static void keep_pool(int device) {
+    static std::mutex mu;
+    static bool done[64] = {false};
+    std::lock_guard<std::mutex> lk(mu);
+    if (device < 0 || device >= 64 || done[device]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    done[device] = true;
+}
+
+static ac_status check_device(int device, cudaDeviceProp *prop) {
+    int count = 0;
+    cudaError_t e = cudaGetDeviceCount(&count);
+    if (e != cudaSuccess || count == 0) {
+        set_error(std::string("no CUDA device: ") + cudaGetErrorString(e));
+        cudaGetLastError();
+        return AC_ERR_NO_DEVICE;
+    }
+    if (device < 0 || device >= count) {
+        set_error("device index out of range");
+        return AC_ERR_INVALID_ARG;
+    }
+    AC_CUDA(cudaGetDeviceProperties(prop, device), "cudaGetDeviceProperties");
+    if (prop->major != 10) {
+        set_error("libac is built for sm_100a only; device is sm_" + std::to_string(prop->major) +
+                  std::to_string(prop->minor));
+        return AC_ERR_NO_DEVICE;
+    }
+    return AC_OK;
+}
+
+static size_t staged_stt_budget(const ac_stt *h) {
+    size_t fixed = staged_smem_bytes(kStaged, 0) + 1024;  // + static smem / slack
+    return h->smem_optin > fixed ? h->smem_optin - fixed : 0;
+}
+
+static SttView view_of(const ac_stt *h) {
+    SttView v;
+    v.stt = h->d_stt;
+    v.cmap = h->d_class_map;
+    v.out_off = h->d_out_off;
+    v.out_ids = h->d_out_ids;
+    v.stride = h->host.row_stride;
+    v.n_states = h->host.n_states;
+    v.smem_rows = h->tier == AC_TIER_GLOBAL ? 0 : h->hot_rows;
+    v.halo = h->host.maxlen ? h->host.maxlen - 1 : 0;
+    return v;
+}
+
+static void free_device(ac_stt *h) {
+    cudaFree(h->d_stt);
+    cudaFree(h->d_class_map);
+    cudaFree(h->d_out_off);
+    cudaFree(h->d_out_ids);
+    cudaFree(h->d_lens);
+    h->d_stt = nullptr;
+    h->d_class_map = nullptr;
+    h->d_out_off = h->d_out_ids = h->d_lens = nullptr;
+}
+
+// ------------------------------------------------------------- the scan
+static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_owned, uint64_t n_halo,
+                             uint64_t base, ac_match_t *d_out, uint64_t cap, ac_result *d_res, cudaStream_t stream,
+                             const ac_match_opts *opts) {
+    g_launches = 0;
+    if (!h || !d_res || (!d_text && n_owned + n_halo > 0)) {
+        set_error("NULL stt, result or text");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (opts && opts->struct_size != sizeof(ac_match_opts)) {
+        set_error("ac_match_opts.struct_size mismatch");
+        return AC_ERR_INVALID_ARG;
+    }
+    const uint64_t n_total = n_owned + n_halo;
+    if (n_total < n_owned || n_total >= AC_MAX_TEXT || base + n_total >= AC_MAX_TEXT) {
+        set_error("text too large (n >= 2^40)");
+        return AC_ERR_TOO_LARGE;
+    }
+    uint32_t kernel = opts ? opts->kernel : AC_KERNEL_AUTO;
+    if (kernel > AC_KERNEL_GLOBAL) {
+        set_error("unknown kernel");
+        return AC_ERR_INVALID_ARG;
+    }
+    const bool emit = d_out != nullptr;
+    void **ev = opts ? opts->events : nullptr;
+    const uint32_t nev = opts ? opts->n_events : 0;
+    auto pre = [&]() {
+        if (ev && g_launches < nev) cudaEventRecord(static_cast<cudaEvent_t>(ev[2 * g_launches]), stream);
+    };
+    auto post = [&](const char *name) {
+        if (ev && g_launches < nev) cudaEventRecord(static_cast<cudaEvent_t>(ev[2 * g_launches + 1]), stream);
+        if (g_launches < 16) g_names[g_launches] = name;
+        g_launches++;
+    };
+    AC_CUDA(cudaMemsetAsync(d_res, 0, sizeof(ac_result), stream), "memset result");
+    if (n_owned == 0 || h->host.n_patterns == 0) return AC_OK;
+
+    const SttView st = view_of(h);
+    const size_t smem_stt = (size_t)st.smem_rows * st.stride * h->host.entry_bytes;
+    const size_t smem_stt16 = (smem_stt + 15) / 16 * 16;
+    const uint32_t eb = h->host.entry_bytes, tier = h->tier;
+    const uint64_t req_chain = opts ? opts->chain_bytes : 0;
+    if (kernel == AC_KERNEL_AUTO) kernel = n_owned >= kStagedMinBytes ? AC_KERNEL_STAGED : AC_KERNEL_GLOBAL;
+
+    // --- geometry: [head | main (staged) | tail] or a single global region
+    Region ra{0, 0, kGlobalTailChain, 0, 0}, rb{0, 0, kGlobalTailChain, 0, 0};
+    StagedGeom g{0, 0, 0, 0, 0};
+    CUtensorMap tmap;
+    if (kernel == AC_KERNEL_STAGED) {
+        const uint64_t W = (uint64_t)kStaged.width, R = (uint64_t)kStaged.threads * kStaged.k;
+        uint64_t head = (16 - (reinterpret_cast<uintptr_t>(d_text) & 15)) & 15;
+        if (head > n_owned) head = n_owned;
+        const uint64_t avail = n_owned - head;
+        uint64_t L;
+        if (req_chain) {
+            L = (req_chain + W - 1) / W * W;
+        } else {
+            const uint64_t target = (uint64_t)h->num_sms * R;
+            L = (avail + target - 1) / target;
+            L = (L + W - 1) / W * W;
+            if (L < kStagedMinChain) L = kStagedMinChain;
+        }
+        if (L > (1ull << 30)) L = (1ull << 30) / W * W;
+        uint64_t n_main = avail / L;
+        if (n_main > (1ull << 31) - R) n_main = ((1ull << 31) - R);
+        ra = Region{0, head, kGlobalTailChain, (head + kGlobalTailChain - 1) / kGlobalTailChain, 0};
+        if (n_main > 0) {
+            g.m0 = head;
+            g.chain_len = L;
+            g.n_chains = n_main;
+            g.chain0 = ra.n_chains;
+            g.n_readable = n_total - head;
+            PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
+            if (!enc) {
+                set_error("cuTensorMapEncodeTiled unavailable from the driver");
+                return AC_ERR_CUDA;
+            }
+            cuuint64_t dims[2] = {(cuuint64_t)L, (cuuint64_t)n_main};
+            cuuint64_t strides[1] = {(cuuint64_t)L};
+            cuuint32_t box[2] = {(cuuint32_t)W, (cuuint32_t)(R < 256 ? R : 256)};
+            cuuint32_t estr[2] = {1, 1};
+            CUresult cr = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, (void *)(d_text + head), dims, strides, box,
+                              estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                              W == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            if (cr != CUDA_SUCCESS) {
+                set_error("cuTensorMapEncodeTiled failed with CUresult " + std::to_string((int)cr));
+                return AC_ERR_CUDA;
+            }
+        }
+        const uint64_t tail_lo = head + n_main * L;
+        rb = Region{tail_lo, n_owned, kGlobalTailChain,
+                    (n_owned - tail_lo + kGlobalTailChain - 1) / kGlobalTailChain, ra.n_chains + n_main};
+    } else {
+        uint64_t L = req_chain;
+        if (!L) {
+            L = (n_owned + (uint64_t)h->num_sms * 1024 - 1) / ((uint64_t)h->num_sms * 1024);
+            L = (L + 15) / 16 * 16;
+            if (L < 64) L = 64;
+        }
+        ra = Region{0, n_owned, L, (n_owned + L - 1) / L, 0};
+    }
+    const uint64_t n_chains = ra.n_chains + g.n_chains + rb.n_chains;
+    const bool any_global = ra.n_chains + rb.n_chains > 0;
+
+    // --- workspace: counts | chain_end | tile_state | counter
+    ScanOut so{};
+    so.base = base;
+    so.res = d_res;
+    so.out = reinterpret_cast<uint64_t *>(d_out);
+    void *ws = nullptr;
+    if (!emit) {
+        so.total = reinterpret_cast<unsigned long long *>(&d_res->count);
+        if (any_global) {
+            pre();
+            AC_CUDA(launch_scan_global(MODE_COUNT_TOTAL, eb, tier, d_text, n_total, st, ra, rb, so, smem_stt16, stream), "k_scan_global(count)");
+            post("k_scan_global(count)");
+        }
+        if (g.n_chains) {
+            pre();
+            AC_CUDA(launch_scan_staged(MODE_COUNT_TOTAL, eb, tier, tmap, d_text + g.m0, st, g, kStaged, so, smem_stt16,
+                                       stream, nullptr), "k_scan_staged(count)");
+            post("k_scan_staged(count)");
+        }
+        return AC_OK;
+    }
+    const size_t tiles = offsets_tiles(n_chains);
+    const size_t bytes = n_chains * 8 * 2 + tiles * 8 + 16;
+    AC_CUDA(cudaMallocAsync(&ws, bytes, stream), "cudaMallocAsync(workspace)");
+    uint64_t *counts = static_cast<uint64_t *>(ws);
+    uint64_t *chain_end = counts + n_chains;
+    uint64_t *tile_state = chain_end + n_chains;
+    unsigned int *counter = reinterpret_cast<unsigned int *>(tile_state + tiles);
+    so.chain_counts = counts;
+    so.chain_end = chain_end;
+    ac_status rc = AC_OK;
+    auto run = [&]() -> ac_status {
+        AC_CUDA(cudaMemsetAsync(tile_state, 0, tiles * 8 + 16, stream), "memset workspace");
+        if (any_global) {
+            pre();
+            AC_CUDA(launch_scan_global(MODE_COUNT_CHAINS, eb, tier, d_text, n_total, st, ra, rb, so, smem_stt16, stream), "k_scan_global(count)");
+            post("k_scan_global(count)");
+        }
+        if (g.n_chains) {
+            pre();
+            AC_CUDA(launch_scan_staged(MODE_COUNT_CHAINS, eb, tier, tmap, d_text + g.m0, st, g, kStaged, so, smem_stt16,
+                                       stream, nullptr), "k_scan_staged(count)");
+            post("k_scan_staged(count)");
+        }
+        pre();
+        AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream), "k_offsets");
+        post("k_offsets");
+        if (any_global) {
+            pre();
+            AC_CUDA(launch_scan_global(MODE_EMIT, eb, tier, d_text, n_total, st, ra, rb, so, smem_stt16, stream), "k_scan_global(emit)");
+            post("k_scan_global(emit)");
+        }
+        if (g.n_chains) {
+            pre();
+            AC_CUDA(launch_scan_staged(MODE_EMIT, eb, tier, tmap, d_text + g.m0, st, g, kStaged, so, smem_stt16, stream,
+                                       nullptr), "k_scan_staged(emit)");
+            post("k_scan_staged(emit)");
+        }
+        return AC_OK;
+    };
+    rc = run();
+    cudaFreeAsync(ws, stream);
+    return rc;
+}
+
+static ac_status finish_sync(ac_result *d_res, uint64_t *count, cudaStream_t stream) {
+    ac_result hres;
+    AC_CUDA(cudaMemcpyAsync(&hres, d_res, sizeof(hres), cudaMemcpyDeviceToHost, stream), "D2H result");
+    AC_CUDA(cudaStreamSynchronize(stream), "cudaStreamSynchronize");
+    if (count) *count = hres.count;
+    if (hres.status != AC_OK) {
+        set_error("match list longer than cap (" + std::to_string(hres.count) + " records needed)");
+        return (ac_status)hres.status;
+    }
+    return AC_OK;
+}
+
+}  // namespace acx
+
+using namespace acx;
+
+extern "C" {
+
+const char *ac_status_string(ac_status s) {
+    switch (s) {
+        case AC_OK: return "AC_OK";
+        case AC_ERR_INVALID_ARG: return "AC_ERR_INVALID_ARG";
+        case AC_ERR_EMPTY_PATTERN: return "AC_ERR_EMPTY_PATTERN";
+        case AC_ERR_TOO_LARGE: return "AC_ERR_TOO_LARGE";
+        case AC_ERR_CAPACITY: return "AC_ERR_CAPACITY";
+        case AC_ERR_NO_MEMORY: return "AC_ERR_NO_MEMORY";
+        case AC_ERR_CUDA: return "AC_ERR_CUDA";
+        case AC_ERR_NO_DEVICE: return "AC_ERR_NO_DEVICE";
+    }
+    return "AC_ERR_UNKNOWN";
+}
+
+const char *ac_last_error(void) { return g_err.c_str(); }
+const char *ac_version(void) { return "libac 0.1 sm_100a (TMA-staged + global-only scans)"; }
+uint32_t ac_last_launch_count(void) { return g_launches; }
+const char *ac_last_launch_name(uint32_t i) { return i < g_launches && i < 16 ? g_names[i] : nullptr; }
+
+ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n, const ac_build_opts *opts,
+                     ac_table **out) {
+    if (!out) {
+        set_error("out is NULL");
+        return AC_ERR_INVALID_ARG;
+    }
+    *out = nullptr;
+    if (opts && opts->struct_size != sizeof(ac_build_opts)) {
+        set_error("ac_build_opts.struct_size mismatch");
+        return AC_ERR_INVALID_ARG;
+    }
+    ac_table *t = new (std::nothrow) ac_table();
+    if (!t) return AC_ERR_NO_MEMORY;
+    ac_status rc;
+    try {
+        rc = compile_table(patterns, lens, n, opts, *t);
+    } catch (...) {
+        set_error("host allocation failed");
+        rc = AC_ERR_NO_MEMORY;
+    }
+    if (rc != AC_OK) {
+        delete t;
+        return rc;
+    }
+    *out = t;
+    return AC_OK;
+}
+
+static void fill_info(const ac_table &t, ac_stt_info *info) {
+    std::memset(info, 0, sizeof(*info));
+    info->n_patterns = t.n_patterns;
+    info->n_states = t.n_states;
+    info->n_classes = t.n_classes;
+    info->row_stride = t.row_stride;
+    info->entry_bytes = t.entry_bytes;
+    info->maxlen = t.maxlen;
+    info->forward = t.forward;
+    info->stt_bytes = (uint64_t)t.n_states * t.row_stride * t.entry_bytes;
+    info->out_entries = t.out_ids.size();
+}
+
+ac_status ac_table_query(const ac_table *t, ac_stt_info *info) {
+    if (!t || !info) return AC_ERR_INVALID_ARG;
+    fill_info(*t, info);
+    return AC_OK;
+}
+
+ac_status ac_table_export(const ac_table *t, uint8_t *class_map, void *stt, uint32_t *out_off, uint32_t *out_ids) {
+    if (!t) return AC_ERR_INVALID_ARG;
+    if (class_map) std::memcpy(class_map, t->class_map, 256);
+    if (stt && !t->stt.empty()) std::memcpy(stt, t->stt.data(), t->stt.size());
+    if (out_off) std::memcpy(out_off, t->out_off.data(), t->out_off.size() * 4);
+    if (out_ids && !t->out_ids.empty()) std::memcpy(out_ids, t->out_ids.data(), t->out_ids.size() * 4);
+    return AC_OK;
+}
+
+void ac_table_free(ac_table *t) { delete t; }
+
+ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n, int device,
+                   const ac_build_opts *opts, ac_stt **out) {
+    if (!out) {
+        set_error("out is NULL");
+        return AC_ERR_INVALID_ARG;
+    }
+    *out = nullptr;
+    if (opts && opts->struct_size != sizeof(ac_build_opts)) {
+        set_error("ac_build_opts.struct_size mismatch");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (opts && opts->forward) {
+        set_error("the device scan needs the reversed automaton (forward=0)");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (opts && opts->tier > AC_TIER_GLOBAL) {
+        set_error("unknown tier");
+        return AC_ERR_INVALID_ARG;
+    }
+    cudaDeviceProp prop;
+    ac_status rc = check_device(device, &prop);
+    if (rc != AC_OK) return rc;
+    ac_stt *h = new (std::nothrow) ac_stt();
+    if (!h) return AC_ERR_NO_MEMORY;
+    try {
+        rc = compile_table(patterns, lens, n, opts, h->host);
+    } catch (...) {
+        rc = AC_ERR_NO_MEMORY;
+    }
+    if (rc != AC_OK) {
+        delete h;
+        return rc;
+    }
+    const ac_table &t = h->host;
+    if ((uint64_t)t.n_states * t.row_stride >= (1ull << 32)) {
+        delete h;
+        set_error("STT has >= 2^32 entries");
+        return AC_ERR_TOO_LARGE;
+    }
+    h->device = device;
+    h->num_sms = prop.multiProcessorCount;
+    h->smem_optin = prop.sharedMemPerBlockOptin;
+    // residency tier
+    const size_t row_bytes = (size_t)t.row_stride * t.entry_bytes;
+    const size_t stt_bytes = (size_t)t.n_states * row_bytes;
+    const size_t budget = staged_stt_budget(h);
+    uint32_t tier = opts ? opts->tier : AC_TIER_AUTO;
+    uint32_t hot = opts ? opts->hot_rows : 0;
+    if (tier == AC_TIER_AUTO) tier = stt_bytes <= budget ? AC_TIER_SMEM : AC_TIER_HYBRID;
+    if (tier == AC_TIER_SMEM) {
+        if (stt_bytes > budget) {
+            delete h;
+            set_error("STT (" + std::to_string(stt_bytes) + " B) does not fit shared memory (" +
+                      std::to_string(budget) + " B)");
+            return AC_ERR_TOO_LARGE;
+        }
+        hot = t.n_states;
+    } else if (tier == AC_TIER_HYBRID) {
+        uint32_t cap_rows = (uint32_t)(budget / row_bytes);
+        if (hot == 0 || hot > cap_rows) hot = cap_rows;
+        if (hot > t.n_states) hot = t.n_states;
+        if (hot == 0) tier = AC_TIER_GLOBAL;
+    } else {
+        hot = 0;
+    }
+    h->tier = tier;
+    h->hot_rows = hot;
+
+    int prev = -1;
+    cudaGetDevice(&prev);
+    auto fail = [&](cudaError_t e, const char *what) {
+        free_device(h);
+        delete h;
+        if (prev >= 0) cudaSetDevice(prev);
+        return e == cudaErrorMemoryAllocation ? (set_error(what), AC_ERR_NO_MEMORY) : cuda_fail(e, what);
+    };
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return fail(e, "cudaSetDevice");
+    const size_t stt_alloc = (stt_bytes + 15) / 16 * 16 + 16;
+    if ((e = cudaMalloc(&h->d_stt, stt_alloc)) != cudaSuccess) return fail(e, "cudaMalloc(stt)");
+    if ((e = cudaMemset(h->d_stt, 0, stt_alloc)) != cudaSuccess) return fail(e, "cudaMemset(stt)");
+    if ((e = cudaMemcpy(h->d_stt, t.stt.data(), stt_bytes, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e, "H2D stt");
+    if ((e = cudaMalloc(&h->d_class_map, 256)) != cudaSuccess) return fail(e, "cudaMalloc(class map)");
+    if ((e = cudaMemcpy(h->d_class_map, t.class_map, 256, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e, "H2D class map");
+    if ((e = cudaMalloc(&h->d_out_off, t.out_off.size() * 4)) != cudaSuccess) return fail(e, "cudaMalloc(out_off)");
+    if ((e = cudaMemcpy(h->d_out_off, t.out_off.data(), t.out_off.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e, "H2D out_off");
+    const size_t nid = t.out_ids.size() ? t.out_ids.size() : 1;
+    if ((e = cudaMalloc(&h->d_out_ids, nid * 4)) != cudaSuccess) return fail(e, "cudaMalloc(out_ids)");
+    if (!t.out_ids.empty() &&
+        (e = cudaMemcpy(h->d_out_ids, t.out_ids.data(), t.out_ids.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e, "H2D out_ids");
+    const size_t nl = t.lens.size() ? t.lens.size() : 1;
+    if ((e = cudaMalloc(&h->d_lens, nl * 4)) != cudaSuccess) return fail(e, "cudaMalloc(lens)");
+    if (!t.lens.empty() && (e = cudaMemcpy(h->d_lens, t.lens.data(), t.lens.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return fail(e, "H2D lens");
+    keep_pool(device);
+    if (prev >= 0 && prev != device) cudaSetDevice(prev);
+    *out = h;
+    return AC_OK;
+}
+
+void ac_free(ac_stt *h) {
+    if (!h) return;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    cudaSetDevice(h->device);
+    free_device(h);
+    if (prev >= 0) cudaSetDevice(prev);
+    delete h;
+}
+
+ac_status ac_stt_query(const ac_stt *h, ac_stt_info *info) {
+    if (!h || !info) return AC_ERR_INVALID_ARG;
+    fill_info(h->host, info);
+    info->tier = h->tier;
+    info->hot_rows = h->hot_rows;
+    return AC_OK;
+}
+
+ac_status ac_stt_pattern_lengths(const ac_stt *h, uint32_t *lens) {
+    if (!h || (!lens && h->host.n_patterns)) return AC_ERR_INVALID_ARG;
+    if (h->host.n_patterns) std::memcpy(lens, h->host.lens.data(), h->host.lens.size() * 4);
+    return AC_OK;
+}
+
+ac_status ac_match_async(const ac_stt *stt, const uint8_t *d_text, uint64_t n_owned, uint64_t n_halo, uint64_t base,
+                         ac_match_t *d_out, uint64_t cap, ac_result *d_result, void *stream,
+                         const ac_match_opts *opts) {
+    try {
+        return match_async(stt, d_text, n_owned, n_halo, base, d_out, cap, d_result,
+                           static_cast<cudaStream_t>(stream), opts);
+    } catch (...) {
+        set_error("unexpected host exception");
+        return AC_ERR_NO_MEMORY;
+    }
+}
+
+ac_status ac_match_shard(const ac_stt *stt, const uint8_t *d_text, uint64_t n_owned, uint64_t n_halo, uint64_t base,
+                         ac_match_t *d_out, uint64_t cap, uint64_t *count, void *stream) {
+    if (!stt) {
+        set_error("stt is NULL");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (n_halo > (stt->host.maxlen ? stt->host.maxlen - 1 : 0)) {
+        set_error("n_halo exceeds maxlen - 1");
+        return AC_ERR_INVALID_ARG;
+    }
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    ac_result *d_res = nullptr;
+    AC_CUDA(cudaMallocAsync(&d_res, sizeof(ac_result), s), "cudaMallocAsync(result)");
+    ac_status rc = ac_match_async(stt, d_text, n_owned, n_halo, base, d_out, cap, d_res, stream, nullptr);
+    if (rc == AC_OK) rc = finish_sync(d_res, count, s);
+    cudaFreeAsync(d_res, s);
+    return rc;
+}
+
+ac_status ac_match(const ac_stt *stt, const uint8_t *d_text, uint64_t n, ac_match_t *d_out, uint64_t cap,
+                   uint64_t *count, void *stream) {
+    return ac_match_shard(stt, d_text, n, 0, 0, d_out, cap, count, stream);
+}
+
+ac_status ac_match_host(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac_match_t *h_out, uint64_t cap,
+                        uint64_t *count, void *stream) {
+    if (!stt || (!h_text && n)) {
+        set_error("NULL stt or text");
+        return AC_ERR_INVALID_ARG;
+    }
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    uint8_t *d_text = nullptr;
+    ac_match_t *d_out = nullptr;
+    ac_result *d_res = nullptr;
+    ac_status rc = AC_OK;
+    auto cleanup = [&]() {
+        if (d_text) cudaFreeAsync(d_text, s);
+        if (d_out) cudaFreeAsync(d_out, s);
+        if (d_res) cudaFreeAsync(d_res, s);
+        cudaStreamSynchronize(s);
+    };
+    cudaError_t e;
+    if ((e = cudaMallocAsync(&d_res, sizeof(ac_result), s)) != cudaSuccess) { cleanup(); return cuda_fail(e, "alloc result"); }
+    if (n && (e = cudaMallocAsync(&d_text, n, s)) != cudaSuccess) { cleanup(); return cuda_fail(e, "alloc text"); }
+    if (h_out && cap && (e = cudaMallocAsync(&d_out, cap * sizeof(ac_match_t), s)) != cudaSuccess) {
+        cleanup();
+        return cuda_fail(e, "alloc out");
+    }
+    if (n && (e = cudaMemcpyAsync(d_text, h_text, n, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
+        cleanup();
+        return cuda_fail(e, "H2D text");
+    }
+    // a NULL h_out means count only; a non-NULL h_out with cap 0 still emits
+    ac_match_t *dst = h_out ? (d_out ? d_out : reinterpret_cast<ac_match_t *>(d_res + 1)) : nullptr;
+    rc = ac_match_async(stt, d_text, n, 0, 0, dst, cap, d_res, stream, nullptr);
+    if (rc == AC_OK) rc = finish_sync(d_res, count, s);
+    if (rc == AC_OK && h_out && count && *count) {
+        if ((e = cudaMemcpyAsync(h_out, d_out, *count * sizeof(ac_match_t), cudaMemcpyDeviceToHost, s)) != cudaSuccess) {
+            cleanup();
+            return cuda_fail(e, "D2H matches");
+        }
+    }
+    cleanup();
+    return rc;
+}
+
+}  // extern "C"

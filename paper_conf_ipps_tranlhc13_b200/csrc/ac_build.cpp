@@ -1,0 +1,205 @@
+// ac_build.cpp -- phase 1 on the host: dictionary -> dense STT.
+//
+// The paper builds "a 2-dimensional matrix (called State Transition Table:
+// STT)" whose rows are DFA states and whose columns are the input symbols,
+// plus a column M flagging matched states (Fig. 5), on a single CPU
+// core.  The DFA's next-move function delta replaces both goto and
+// failure functions.  What differs here:
+//
+//   * Alphabet compaction: the 256 byte columns collapse to C classes; class
+//     0 = every byte that occurs in no pattern (its column is all-root), the
+//     others are the bytes that occur, in byte order.
+//   * Orientation: by default the automaton is built over the REVERSED
+//     patterns and the scan walks right to left, so a state's output set is
+//     the set of patterns STARTING at the current position and the matches
+//     leave each chain already in canonical (start, pattern) order.  The
+//     forward (paper) orientation is kept for builder tests.
+//   * Column M is folded into each entry: the top bit of delta(s,c) says
+//     "output(delta(s,c)) is non-empty" (reading R10), so the hot loop
+//     learns about a match from the same load that moves it.
+//   * BFS state numbering: shallow (hot) states form a prefix of the table,
+//     which is what a shared-memory hot prefix keeps resident.
+//   * Rows are padded to an odd number of 4-byte words (bank spreading).
+//   * output(s) is stored as CSR with ids ascending (the closure over the
+//     failure function).
+//
+// Construction is the textbook one (AC'75 Alg. 2-4) on a dense goto table.
+#include <algorithm>
+#include <cstring>
+#include <deque>
+#include <new>
+
+#include "ac_internal.h"
+
+namespace acx {
+
+ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n,
+                        const ac_build_opts *opts, ac_table &t) {
+    if (n > 0 && (!patterns || !lens)) {
+        set_error("patterns/lens is NULL");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (n >= AC_MAX_PATTERNS) {
+        set_error("n_patterns must be < 2^24");
+        return AC_ERR_TOO_LARGE;
+    }
+    uint32_t want_eb = opts ? opts->entry_bytes : 0;
+    if (want_eb != 0 && want_eb != 2 && want_eb != 4) {
+        set_error("entry_bytes must be 0, 2 or 4");
+        return AC_ERR_INVALID_ARG;
+    }
+    t.forward = opts ? (opts->forward ? 1u : 0u) : 0u;
+    t.n_patterns = n;
+    t.lens.assign(lens, lens + n);
+    uint64_t total = 0;
+    t.maxlen = 0;
+    bool used[256] = {false};
+    for (uint32_t p = 0; p < n; p++) {
+        if (lens[p] == 0) {
+            set_error("pattern " + std::to_string(p) + " is empty");
+            return AC_ERR_EMPTY_PATTERN;
+        }
+        if (!patterns[p]) {
+            set_error("patterns[" + std::to_string(p) + "] is NULL");
+            return AC_ERR_INVALID_ARG;
+        }
+        t.maxlen = std::max(t.maxlen, lens[p]);
+        total += lens[p];
+        for (uint32_t j = 0; j < lens[p]; j++) used[patterns[p][j]] = true;
+    }
+    if (total + 1 >= (1ull << 31)) {
+        set_error("too many states");
+        return AC_ERR_TOO_LARGE;
+    }
+    // ---- alphabet classes
+    uint32_t C = 1;
+    for (int b = 0; b < 256; b++) t.class_map[b] = 0;
+    for (int b = 0; b < 256; b++)
+        if (used[b]) t.class_map[b] = (uint8_t)std::min<uint32_t>(C++, 255);
+    // C can reach 257 when every byte occurs; class ids then need 9 bits.
+    // We keep class 0 only if some byte is unused: with all 256 bytes used the
+    // map is the identity shifted by one, which would overflow uint8, so map
+    // byte b -> b and drop the empty class.
+    if (C == 257) {
+        for (int b = 0; b < 256; b++) t.class_map[b] = (uint8_t)b;
+        C = 256;
+    }
+    t.n_classes = C;
+
+    try {
+        // ---- goto function (AC'75 Alg. 2) on a dense table, creation order
+        std::vector<int32_t> go;
+        go.reserve((size_t)std::min<uint64_t>(total + 1, 1u << 22) * C);
+        go.assign(C, -1);
+        std::vector<std::vector<uint32_t>> own(1);
+        uint32_t S = 1;
+        for (uint32_t p = 0; p < n; p++) {
+            uint32_t s = 0;
+            for (uint32_t j = 0; j < lens[p]; j++) {
+                uint8_t b = t.forward ? patterns[p][j] : patterns[p][lens[p] - 1 - j];
+                uint32_t c = t.class_map[b];
+                int32_t nx = go[(size_t)s * C + c];
+                if (nx < 0) {
+                    nx = (int32_t)S++;
+                    go[(size_t)s * C + c] = nx;
+                    go.insert(go.end(), C, -1);
+                    own.emplace_back();
+                }
+                s = (uint32_t)nx;
+            }
+            own[s].push_back(p);
+        }
+        // ---- BFS order, failure function and delta (AC'75 Alg. 3/4)
+        std::vector<uint32_t> order;
+        order.reserve(S);
+        std::vector<uint32_t> fail(S, 0);
+        std::vector<uint8_t> is_child(C);
+        order.push_back(0);
+        for (size_t qi = 0; qi < order.size(); qi++) {
+            uint32_t r = order[qi];
+            int32_t *row = &go[(size_t)r * C];
+            for (uint32_t c = 0; c < C; c++) {
+                int32_t child = row[c];
+                if (child >= 0) {
+                    order.push_back((uint32_t)child);
+                    fail[child] = (r == 0) ? 0u : (uint32_t)(go[(size_t)fail[r] * C + c] & 0x7fffffff);
+                    row[c] = child;
+                } else {
+                    // delta(r,c) = delta(f(r),c); the root loops to itself
+                    row[c] = (r == 0) ? 0 : go[(size_t)fail[r] * C + c];
+                }
+            }
+        }
+        // after this loop go[] holds delta (all entries >= 0)
+        // ---- output closure, in BFS order (f(s) is shallower than s)
+        std::vector<std::vector<uint32_t>> out(S);
+        for (uint32_t s : order) {
+            std::vector<uint32_t> v = own[s];
+            if (s != 0) {
+                const std::vector<uint32_t> &fo = out[fail[s]];
+                v.insert(v.end(), fo.begin(), fo.end());
+            }
+            std::sort(v.begin(), v.end());
+            out[s].swap(v);
+        }
+        own.clear();
+        own.shrink_to_fit();
+        // ---- renumber in BFS order
+        std::vector<uint32_t> rank(S);
+        for (uint32_t i = 0; i < S; i++) rank[order[i]] = i;
+        uint32_t eb = want_eb ? want_eb : (S <= 32768 ? 2u : 4u);
+        if (eb == 2 && S > 32768) {
+            set_error("entry_bytes=2 needs <= 32768 states");
+            return AC_ERR_TOO_LARGE;
+        }
+        // odd number of 4-byte words per row
+        uint32_t stride;
+        if (eb == 2) {
+            uint32_t words = (C + 1) / 2;
+            if (words % 2 == 0) words++;
+            stride = words * 2;
+        } else {
+            stride = C | 1u;
+        }
+        t.n_states = S;
+        t.row_stride = stride;
+        t.entry_bytes = eb;
+        t.stt.assign((size_t)S * stride * eb, 0);
+        t.out_off.assign(S + 1, 0);
+        uint64_t n_out = 0;
+        for (uint32_t i = 0; i < S; i++) {
+            t.out_off[i] = (uint32_t)n_out;
+            n_out += out[order[i]].size();
+            if (n_out >= (1ull << 32)) {
+                set_error("output closure too large");
+                return AC_ERR_TOO_LARGE;
+            }
+        }
+        t.out_off[S] = (uint32_t)n_out;
+        t.out_ids.resize(n_out);
+        for (uint32_t i = 0; i < S; i++) {
+            const std::vector<uint32_t> &v = out[order[i]];
+            std::copy(v.begin(), v.end(), t.out_ids.begin() + t.out_off[i]);
+        }
+        for (uint32_t i = 0; i < S; i++) {
+            const int32_t *row = &go[(size_t)order[i] * C];
+            for (uint32_t c = 0; c < C; c++) {
+                uint32_t nx = rank[(uint32_t)row[c]];
+                bool flag = !out[(uint32_t)row[c]].empty();
+                if (eb == 2) {
+                    uint16_t e = (uint16_t)(nx | (flag ? 0x8000u : 0u));
+                    std::memcpy(&t.stt[((size_t)i * stride + c) * 2], &e, 2);
+                } else {
+                    uint32_t e = nx | (flag ? 0x80000000u : 0u);
+                    std::memcpy(&t.stt[((size_t)i * stride + c) * 4], &e, 4);
+                }
+            }
+        }
+    } catch (const std::bad_alloc &) {
+        set_error("host allocation failed while building the STT");
+        return AC_ERR_NO_MEMORY;
+    }
+    return AC_OK;
+}
+
+}  // namespace acx

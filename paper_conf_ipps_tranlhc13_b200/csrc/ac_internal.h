@@ -1,0 +1,45 @@
+// ac_internal.h -- internal types of libac (not part of the ABI).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "ac.h"
+
+// Phase-1 result on the host (P:118 STT, P:137 built once on the host).
+struct ac_table {
+    uint32_t n_patterns = 0;
+    uint32_t maxlen = 0;
+    uint32_t n_states = 0;
+    uint32_t n_classes = 0;
+    uint32_t row_stride = 0;   // entries per row
+    uint32_t entry_bytes = 2;
+    uint32_t forward = 0;
+    uint8_t class_map[256] = {0};
+    std::vector<uint8_t> stt;          // n_states * row_stride * entry_bytes
+    std::vector<uint32_t> out_off;     // n_states + 1
+    std::vector<uint32_t> out_ids;     // output CSR (ids ascending per state)
+    std::vector<uint32_t> lens;        // pattern lengths
+};
+
+// Device-side STT (library owned).
+struct ac_stt {
+    ac_table host;        // keeps the host copy for query / re-upload
+    int device = 0;
+    uint32_t tier = AC_TIER_GLOBAL;
+    uint32_t hot_rows = 0;
+    void *d_stt = nullptr;           // entries
+    uint8_t *d_class_map = nullptr;  // 256 B
+    uint32_t *d_out_off = nullptr;
+    uint32_t *d_out_ids = nullptr;
+    uint32_t *d_lens = nullptr;
+    int num_sms = 148;
+    size_t smem_optin = 227 * 1024;
+};
+
+namespace acx {
+void set_error(const std::string &msg);
+ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n,
+                        const ac_build_opts *opts, ac_table &t);
+}  // namespace acx

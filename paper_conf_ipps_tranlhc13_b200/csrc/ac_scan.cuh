@@ -1,0 +1,76 @@
+// ac_scan.cuh -- launch interface between the ABI layer and the scan kernels.
+#pragma once
+
+#include <cstdint>
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include "ac.h"
+
+namespace acx {
+
+enum ScanMode { MODE_COUNT_TOTAL = 0, MODE_COUNT_CHAINS = 1, MODE_EMIT = 2 };
+
+// Read-only automaton as the kernels see it.
+struct SttView {
+    const void *stt;          // entries, row-major, row_stride entries per row
+    const uint8_t *cmap;      // byte -> class (256 B)
+    const uint32_t *out_off;  // output CSR offsets [S + 1]
+    const uint32_t *out_ids;  // output CSR ids (ascending per state)
+    uint32_t stride;          // entries per row
+    uint32_t n_states;
+    uint32_t smem_rows;       // rows staged into shared memory
+    uint32_t halo;            // maxlen - 1
+};
+
+// A run of equal-length chains over owned starts [lo, hi) of the shard.
+struct Region {
+    uint64_t lo, hi;       // owned byte range (shard coordinates)
+    uint64_t chain_len;    // bytes owned per chain (last chain may be shorter)
+    uint64_t n_chains;
+    uint64_t chain0;       // global index of the region's first chain
+};
+
+// Where results go.
+struct ScanOut {
+    unsigned long long *total;      // MODE_COUNT_TOTAL: atomic sum
+    uint64_t *chain_counts;         // MODE_COUNT_CHAINS
+    const uint64_t *chain_end;      // MODE_EMIT: inclusive prefix (end offset) per chain
+    const ac_result *res;           // MODE_EMIT: skip writing when res->status != AC_OK
+    uint64_t *out;                  // MODE_EMIT: records
+    uint64_t base;                  // global position of shard byte 0
+};
+
+// Geometry of the TMA-staged main region.
+struct StagedGeom {
+    uint64_t m0;           // shard offset of the main region (16-byte aligned address)
+    uint64_t chain_len;    // L, multiple of the tile width
+    uint64_t n_chains;     // full chains in the main region
+    uint64_t chain0;       // global index of main chain 0
+    uint64_t n_readable;   // bytes readable from the main-region pointer (halo bound)
+};
+
+struct StagedConfig {
+    int threads;     // CTA size
+    int k;           // chains per thread
+    int width;       // tile width S in bytes (64 or 128, = TMA swizzle span)
+    int stages;      // ring depth
+};
+
+// Kernel entry points (host side launchers); all return cudaError_t.
+cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,
+                               uint64_t n_total, const SttView &st, const Region &a, const Region &b,
+                               const ScanOut &so, size_t smem_bytes, cudaStream_t stream);
+cudaError_t launch_scan_staged(int mode, uint32_t entry_bytes, uint32_t tier, const CUtensorMap &tmap,
+                               const uint8_t *main_text, const SttView &st, const StagedGeom &g,
+                               const StagedConfig &cfg, const ScanOut &so, size_t smem_stt_bytes,
+                               cudaStream_t stream, int *ctas_out);
+cudaError_t launch_offsets(const uint64_t *counts, uint64_t n, uint64_t *chain_end, uint64_t *tile_state,
+                           unsigned int *tile_counter, ac_result *res, uint64_t cap, int emitting,
+                           cudaStream_t stream);
+
+size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
+size_t offsets_tiles(uint64_t n);
+
+}  // namespace acx

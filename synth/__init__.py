@@ -36,22 +36,23 @@ def rng_for(seed: int, j: int = 0) -> np.random.Generator:
     return np.random.Generator(np.random.PCG64(splitmix64((seed ^ j) & MASK64)))
 
 
-def _blocks(n: int, seed: int, fill) -> np.ndarray:
-    """Allocate n bytes and fill them block by block with fill(rng, view, j)."""
+def _blocks(n: int, seed: int, fill, block0: int = 0) -> np.ndarray:
+    """Allocate n bytes and fill them block by block with fill(rng, view, j);
+    the text starts at block ``block0`` of the (endless) seeded stream."""
     out = np.empty(n, dtype=np.uint8)
     for j, lo in enumerate(range(0, n, BLOCK)):
         hi = min(n, lo + BLOCK)
-        fill(rng_for(seed, j), out[lo:hi], j)
+        fill(rng_for(seed, block0 + j), out[lo:hi], block0 + j)
     return out
 
 
 # ---------------------------------------------------------------------------
 # C1: iid lowercase text, iid lowercase patterns
 # ---------------------------------------------------------------------------
-def text_lowercase(n: int, seed: int) -> np.ndarray:
+def text_lowercase(n: int, seed: int, block0: int = 0) -> np.ndarray:
     def fill(rng, v, j):
         v[:] = rng.integers(ord("a"), ord("z") + 1, size=v.size, dtype=np.uint8)
-    return _blocks(n, seed, fill)
+    return _blocks(n, seed, fill, block0)
 
 
 def patterns_random(count: int, lmin: int, lmax: int, seed: int, alphabet: bytes) -> list[bytes]:
@@ -89,7 +90,8 @@ def english_vocabulary(seed: int, words: int = 20000, mean_len: float = 5.0, max
     return Vocabulary(flat, off, lens, cdf)
 
 
-def text_english(n: int, seed: int, vocab: Vocabulary, punct: float = 0.05, words_per_line: int = 12) -> np.ndarray:
+def text_english(n: int, seed: int, vocab: Vocabulary, punct: float = 0.05, words_per_line: int = 12,
+                 block0: int = 0) -> np.ndarray:
     def fill(rng, v, j):
         pos = 0
         while pos < v.size:
@@ -111,7 +113,7 @@ def text_english(n: int, seed: int, vocab: Vocabulary, punct: float = 0.05, word
             take = min(total, v.size - pos)
             v[pos:pos + take] = buf[:take]
             pos += take
-    return _blocks(n, seed, fill)
+    return _blocks(n, seed, fill, block0)
 
 
 def patterns_substrings(text: np.ndarray, count: int, lmin: int, lmax: int, seed: int) -> list[bytes]:
@@ -139,7 +141,7 @@ def patterns_snort(count: int, seed: int, mean_extra: float = 11.0, lmin: int = 
 
 
 def text_payload(n: int, seed: int, patterns: list[bytes], chunk: int = 64,
-                 p_printable: float = 0.60, p_planted: float = 0.02) -> np.ndarray:
+                 p_printable: float = 0.60, p_planted: float = 0.02, block0: int = 0) -> np.ndarray:
     pat_flat = np.frombuffer(b"".join(patterns), dtype=np.uint8)
     pat_len = np.array([len(p) for p in patterns], dtype=np.int64)
     pat_off = np.concatenate([[0], np.cumsum(pat_len)[:-1]])
@@ -160,7 +162,7 @@ def text_payload(n: int, seed: int, patterns: list[bytes], chunk: int = 64,
             dst = np.repeat(planted * chunk + off, L) + within
             buf[dst] = pat_flat[np.repeat(pat_off[pid], L) + within]
         v[:] = buf[:v.size]
-    return _blocks(n, seed, fill)
+    return _blocks(n, seed, fill, block0)
 
 
 # ---------------------------------------------------------------------------
@@ -169,7 +171,7 @@ def text_payload(n: int, seed: int, patterns: list[bytes], chunk: int = 64,
 _ACGT = np.frombuffer(b"ACGT", dtype=np.uint8)
 
 
-def text_dna(n: int, seed: int, p_n_run: float = 1e-4, max_run: int = 100) -> np.ndarray:
+def text_dna(n: int, seed: int, p_n_run: float = 1e-4, max_run: int = 100, block0: int = 0) -> np.ndarray:
     def fill(rng, v, j):
         v[:] = _ACGT[rng.integers(0, 4, size=v.size, dtype=np.uint8)]
         k = rng.binomial(v.size, p_n_run)
@@ -179,7 +181,7 @@ def text_dna(n: int, seed: int, p_n_run: float = 1e-4, max_run: int = 100) -> np
             within = np.arange(int(L.sum())) - np.repeat(np.cumsum(L) - L, L)
             idx = np.repeat(st, L) + within
             v[idx[idx < v.size]] = ord("N")
-    return _blocks(n, seed, fill)
+    return _blocks(n, seed, fill, block0)
 
 
 def patterns_kmers(text: np.ndarray, count: int, seed: int, lmin: int = 20, lmax: int = 32,
@@ -229,6 +231,31 @@ class Workload:
 
 
 C_SIZES = {"c1": 1 << 20, "c2": 1 << 28, "c3": 1 << 30, "c4": 1 << 32}
+
+
+def stream(w: Workload, name: str, block0: int, nbytes: int) -> np.ndarray:
+    """nbytes of config `name`'s endless text stream starting at block0."""
+    m = (nbytes + BLOCK - 1) // BLOCK * BLOCK
+    b0 = block0
+    if name == "c1":
+        t = text_lowercase(m, 1000, b0)
+    elif name == "c2":
+        t = text_english(m, 2000, english_vocabulary(2002), block0=b0)
+    elif name == "c3":
+        t = text_payload(m, 3000, w.patterns, block0=b0)
+    elif name == "c4":
+        t = text_dna(m, 4000, block0=b0)
+    else:
+        raise ValueError(name)
+    return t[:nbytes]
+
+
+def segment(w: Workload, name: str, index: int, n: int, extra: int) -> np.ndarray:
+    """Bytes [index*n, (index+1)*n + extra) of config `name`'s text stream
+    (n a multiple of BLOCK): rank `index`'s shard plus its halo, for the
+    weak-scaled multi-GPU bench.  Segment 0 without extra is w.text."""
+    assert n % BLOCK == 0
+    return stream(w, name, index * (n // BLOCK), n + extra)
 
 
 def make(name: str, n: int | None = None, n_patterns: int | None = None) -> Workload:

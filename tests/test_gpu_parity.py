@@ -1,0 +1,330 @@
+"""GPU parity: libac's sm_100a scan against the CPU oracle, record by record.
+
+Bar: bit-exact -- identical canonical lists (start, pattern) and counts
+(integer work).  Inputs are the seeded synthetic workloads of synth/, at
+oracle-sized scales that still span many CTA tiles and ragged tails, plus the
+full BASELINE.json sizes in the launch configuration bench.py times, checked
+on sampled windows (oracle.match_window) and closed forms.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_ipps_tranlhc13_b200 as ac
+import synth
+from oracle import Oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _gpu():
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    ac.build_library()
+    ac.lib()
+
+
+def oracle_keys(o: Oracle, text, lo=None, hi=None) -> np.ndarray:
+    if lo is None:
+        ends, pids = o.match(text)
+    else:
+        ends, pids = o.match_window(text, lo, hi)
+    starts = ends.astype(np.int64) - o.lens[pids].astype(np.int64) + 1
+    return (starts << 24) | pids.astype(np.int64)
+
+
+def gpu_keys(stt, text_np: np.ndarray, **kw) -> np.ndarray:
+    t = torch.from_numpy(np.ascontiguousarray(text_np)).cuda() if text_np.size else torch.empty(0, dtype=torch.uint8, device="cuda")
+    c, recs = ac.match(stt, t, **kw)
+    cnt = ac.count(stt, t, **{k: v for k, v in kw.items() if k in ("kernel", "chain_bytes")})
+    assert cnt == c
+    return recs.cpu().numpy()
+
+
+def assert_same(got: np.ndarray, want: np.ndarray):
+    assert got.shape == want.shape, (got.shape, want.shape)
+    if got.size:
+        bad = np.nonzero(got != want)[0]
+        assert bad.size == 0, f"first mismatch at {bad[0]}: got {got[bad[0]]:#x} want {want[bad[0]]:#x}"
+
+
+KERNELS = [ac.KERNEL_STAGED, ac.KERNEL_GLOBAL]
+
+
+# ----------------------------------------------------------------- examples
+def test_worked_example():
+    pats = [b"he", b"she", b"his", b"hers"]
+    stt = ac.build(pats)
+    for k in KERNELS:
+        got = gpu_keys(stt, np.frombuffer(b"ushers", np.uint8), kernel=k)
+        # she@1, he@2, hers@2 (north_star)
+        assert [(int(x) >> 24, pats[int(x) & 0xFFFFFF]) for x in got] == [(1, b"she"), (2, b"he"), (2, b"hers")]
+        e = ac.ends(torch.from_numpy(got), stt.lens).tolist()
+        assert e == [3, 3, 5]
+
+
+# ---------------------------------------------------------- configs (scaled)
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_c1_full(kernel):
+    w = synth.make("c1")
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    assert stt.tier_name == "smem"
+    assert_same(gpu_keys(stt, w.text, kernel=kernel), oracle_keys(o, w.text))
+
+
+@pytest.mark.parametrize("name,n", [("c2", 3 << 20), ("c3", 1 << 20), ("c4", 3 << 20)])
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_configs_scaled(name, n, kernel):
+    w = synth.make(name, n=n + 12345)  # ragged tail
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    assert_same(gpu_keys(stt, w.text, kernel=kernel), oracle_keys(o, w.text))
+
+
+@pytest.mark.parametrize("tier,hot,eb", [(ac.TIER_SMEM, 0, 2), (ac.TIER_HYBRID, 37, 2), (ac.TIER_GLOBAL, 0, 2),
+                                         (ac.TIER_SMEM, 0, 4), (ac.TIER_HYBRID, 5, 4), (ac.TIER_GLOBAL, 0, 4)])
+def test_tiers_and_widths(tier, hot, eb):
+    w = synth.make("c2", n=(1 << 20) + 77, n_patterns=60)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns, tier=tier, hot_rows=hot, entry_bytes=eb)
+    assert stt.info["tier"] == tier and stt.info["entry_bytes"] == eb
+    want = oracle_keys(o, w.text)
+    for k in KERNELS:
+        assert_same(gpu_keys(stt, w.text, kernel=k), want)
+
+
+def test_c3_hybrid_and_global_tiers():
+    w = synth.make("c3", n=(1 << 20) + 5)
+    o = Oracle(w.patterns)
+    want = oracle_keys(o, w.text)
+    for tier in (ac.TIER_AUTO, ac.TIER_GLOBAL):
+        stt = ac.build(w.patterns, tier=tier)
+        assert_same(gpu_keys(stt, w.text), want)
+
+
+@pytest.mark.parametrize("chain", [64, 128, 320, 1024, 4096, 65536])
+def test_chunking_invariance_staged(chain):
+    w = synth.make("c2", n=(2 << 20) + 999, n_patterns=300)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, chain_bytes=chain), oracle_keys(o, w.text))
+
+
+@pytest.mark.parametrize("chain", [1, 7, 16, 64, 1000, 1 << 20])
+def test_chunking_invariance_global(chain):
+    w = synth.make("c1", n=(1 << 18) + 3)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_GLOBAL, chain_bytes=chain), oracle_keys(o, w.text))
+
+
+# --------------------------------------------------------------- edge cases
+def test_empty_and_short_texts():
+    pats = [b"abc", b"b", b"abcdefgh"]
+    o = Oracle(pats)
+    stt = ac.build(pats)
+    for t in [b"", b"a", b"b", b"ab", b"abc", b"abcdefg", b"abcdefgh"]:
+        arr = np.frombuffer(t, np.uint8)
+        for k in KERNELS:
+            assert_same(gpu_keys(stt, arr, kernel=k), oracle_keys(o, arr))
+
+
+def test_boundary_straddling_everywhere():
+    rng = np.random.default_rng(11)
+    pats = [b"0123456789abcdefghijklmnopqrstuvwxyz"[:L] for L in (2, 5, 17, 31, 36)] + [b"Z"]
+    text = rng.integers(ord("A"), ord("Y"), size=(1 << 20) + 333, dtype=np.uint8)
+    p = np.frombuffer(pats[4], np.uint8)
+    for chain in (256, 1024):
+        for boundary in range(chain, text.size - 64, chain * 7):
+            j = int(rng.integers(0, p.size))
+            text[boundary - j: boundary - j + p.size] = p
+    text[:p.size] = p
+    text[-p.size:] = p
+    o = Oracle(pats)
+    want = oracle_keys(o, text)
+    stt = ac.build(pats)
+    for chain in (256, 1024):
+        assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED, chain_bytes=chain), want)
+        assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_GLOBAL, chain_bytes=chain // 4), want)
+
+
+def test_all_byte_values_and_nul():
+    rng = np.random.default_rng(3)
+    text = rng.integers(0, 256, size=(1 << 19) + 1, dtype=np.uint8)
+    text[1000:1010] = 0
+    pats = [bytes([b]) for b in range(0, 256, 5)] + [b"\x00\x00\x00", text[5000:5009].tobytes(), b"\xff\x00"]
+    o = Oracle(pats)
+    want = oracle_keys(o, text)
+    stt = ac.build(pats)
+    assert stt.maxlen == 9
+    for k in KERNELS:
+        assert_same(gpu_keys(stt, text, kernel=k), want)
+
+
+def test_single_byte_patterns_no_halo():
+    text = np.frombuffer(b"abracadabra" * 20000, np.uint8)
+    pats = [b"a", b"r", b"a"]
+    o = Oracle(pats)
+    stt = ac.build(pats)
+    assert stt.maxlen == 1
+    for k in KERNELS:
+        assert_same(gpu_keys(stt, text, kernel=k), oracle_keys(o, text))
+
+
+def test_no_pattern_bytes():
+    stt = ac.build([b"xyz", b"q"])
+    t = torch.full((1 << 20,), ord("a"), dtype=torch.uint8, device="cuda")
+    assert ac.count(stt, t) == 0
+    c, recs = ac.match(stt, t)
+    assert c == 0 and recs.numel() == 0
+
+
+def test_duplicates_and_nested():
+    pats = [b"ab", b"ab", b"b", b"abab", b"bab", b"ababababab"]
+    text = np.frombuffer(b"xababab" * 30000 + b"ab", np.uint8)
+    o = Oracle(pats)
+    stt = ac.build(pats)
+    for k in KERNELS:
+        assert_same(gpu_keys(stt, text, kernel=k), oracle_keys(o, text))
+
+
+@pytest.mark.parametrize("n", [31, 1 << 16, (1 << 20) + 17])
+def test_adversarial_runs_closed_form(n):
+    K = 32
+    pats = [b"a" * k for k in range(1, K + 1)]
+    stt = ac.build(pats)
+    t = torch.full((n,), ord("a"), dtype=torch.uint8, device="cuda")
+    want_count = K * n - K * (K - 1) // 2 if n >= K else n * (n + 1) // 2
+    for k in KERNELS:
+        assert ac.count(stt, t, kernel=k) == want_count
+        c, recs = ac.match(stt, t, kernel=k)
+        assert c == want_count
+        r = recs.cpu().numpy()
+        s = r >> 24
+        p = r & 0xFFFFFF
+        # start-major, pattern ids ascending, pattern p (length p+1) fits
+        exp_s = np.repeat(np.arange(n), np.minimum(K, n - np.arange(n)))
+        assert np.array_equal(s, exp_s)
+        first = np.concatenate([[True], s[1:] != s[:-1]])
+        exp_p = np.arange(r.size) - np.maximum.accumulate(np.where(first, np.arange(r.size), 0))
+        assert np.array_equal(p, exp_p)
+
+
+@pytest.mark.parametrize("off", [1, 3, 7, 8, 13, 15])
+def test_misaligned_text_pointer(off):
+    w = synth.make("c2", n=(1 << 20) + 100, n_patterns=200)
+    o = Oracle(w.patterns)
+    big = torch.from_numpy(w.text).cuda()
+    sub = big[off:]
+    assert sub.data_ptr() % 16 == off % 16
+    c, recs = ac.match(ac.build(w.patterns), sub, kernel=ac.KERNEL_STAGED)
+    assert_same(recs.cpu().numpy(), oracle_keys(o, w.text[off:]))
+
+
+def test_capacity_error_and_count_only():
+    w = synth.make("c1", n=1 << 18)
+    stt = ac.build(w.patterns)
+    t = torch.from_numpy(w.text).cuda()
+    need = ac.count(stt, t)
+    assert need > 10
+    out = torch.empty(need - 1, dtype=torch.int64, device="cuda")
+    with pytest.raises(ac.CapacityError) as e:
+        ac.match(stt, t, out)
+    assert e.value.count == need
+    out = torch.empty(need, dtype=torch.int64, device="cuda")
+    c, _ = ac.match(stt, t, out)
+    assert c == need
+
+
+def test_shard_api_concatenation():
+    w = synth.make("c2", n=(3 << 20) + 11, n_patterns=400)
+    o = Oracle(w.patterns)
+    want = oracle_keys(o, w.text)
+    stt = ac.build(w.patterns)
+    t = torch.from_numpy(w.text).cuda()
+    n = t.numel()
+    rng = np.random.default_rng(1)
+    for G in (2, 3, 8):
+        cuts = np.sort(rng.integers(0, n, size=G - 1)).tolist()
+        bounds = [0] + cuts + [n]
+        parts = []
+        for lo, hi in zip(bounds[:-1], bounds[1:]):
+            halo = min(stt.maxlen - 1, n - hi)
+            c, recs = ac.match(stt, t[lo:hi + halo], n_halo=halo, base=lo)
+            parts.append(recs.cpu().numpy())
+        assert_same(np.concatenate(parts), want)
+
+
+def test_host_entry_point():
+    w = synth.make("c1", n=(1 << 18) + 5)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    host = torch.from_numpy(w.text).pin_memory()
+    want = oracle_keys(o, w.text)
+    out = torch.empty(want.size + 10, dtype=torch.int64).pin_memory()
+    c = ac.match_host(stt, host, out)
+    assert c == want.size
+    assert_same(out[:c].numpy(), want)
+    assert ac.match_host(stt, host, None) == want.size
+
+
+def test_determinism():
+    w = synth.make("c2", n=(2 << 20) + 1, n_patterns=500)
+    stt = ac.build(w.patterns)
+    t = torch.from_numpy(w.text).cuda()
+    a = ac.match(stt, t)[1].cpu().numpy()
+    b = ac.match(stt, t)[1].cpu().numpy()
+    assert np.array_equal(a, b)
+
+
+# ------------------------------------------------- full BASELINE.json sizes
+def _windows(n, k, width, seed):
+    rng = np.random.default_rng(seed)
+    los = [0, n - width] + rng.integers(0, n - width, size=k - 2).tolist()
+    return [(int(lo), int(lo) + width) for lo in los]
+
+
+def _check_windows(o, text_np, recs_np, windows):
+    s = recs_np >> 24
+    for lo, hi in windows:
+        a, b = np.searchsorted(s, lo, "left"), np.searchsorted(s, hi, "left")
+        assert_same(recs_np[a:b], oracle_keys(o, text_np, lo, hi))
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name,width,k", [("c2", 1 << 18, 8), ("c3", 1 << 17, 5), ("c4", 1 << 18, 6)])
+def test_full_size_sampled(name, width, k):
+    w = synth.make(name)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    t = torch.from_numpy(w.text).cuda()
+    c, recs = ac.match(stt, t)
+    r = recs.cpu().numpy()
+    assert c == r.size and (c == 0 or np.all(r[1:] > r[:-1]))  # canonical and duplicate free
+    # count-only agrees with the list; the staged and global-only kernels agree
+    assert ac.count(stt, t) == c
+    _check_windows(o, w.text, r, _windows(w.text.size, k, width, 7))
+    del t, recs
+
+
+@pytest.mark.slow
+def test_full_size_closed_form_kmers():
+    # all 4^6 6-mers over ACGT, ids lexicographic: one match per start, pid =
+    # base-4 value of text[i:i+6] (closed form P4-ii, exact at any size)
+    A = b"ACGT"
+    import itertools
+    pats = [bytes(t) for t in itertools.product(A, repeat=6)]
+    n = 1 << 30
+    digits = synth.rng_for(424242).integers(0, 4, size=n, dtype=np.uint8)
+    text = np.frombuffer(A, np.uint8)[digits]
+    stt = ac.build(pats)
+    c, recs = ac.match(stt, torch.from_numpy(text).cuda())
+    assert c == n - 5
+    r = recs.cpu().numpy()
+    assert np.array_equal(r >> 24, np.arange(n - 5))
+    d = digits.astype(np.int64)
+    val = d[:-5] * 1024 + d[1:-4] * 256 + d[2:-3] * 64 + d[3:-2] * 16 + d[4:-1] * 4 + d[5:]
+    assert np.array_equal(r & 0xFFFFFF, val)

@@ -1,0 +1,171 @@
+"""CPU tests of libac: the library loads and exports every symbol of
+include/ac.h, the host builder (phase 1) equals the oracle's
+goto/failure/output definitions state by state, and the device entry points
+fail loudly without a GPU (no CPU fallback)."""
+from __future__ import annotations
+
+import ctypes
+import random
+import re
+from pathlib import Path
+
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_ipps_tranlhc13_b200 as ac
+from oracle import Oracle
+
+ROOT = Path(__file__).resolve().parents[1]
+
+
+@pytest.fixture(scope="session", autouse=True)
+def _built():
+    ac.build_library()
+
+
+def test_exports_every_declared_symbol():
+    header = (ROOT / "include" / "ac.h").read_text()
+    declared = set(re.findall(r"^\s*(?:const\s+)?[\w\s\*]+?\b(ac_\w+)\s*\(", header, re.M))
+    declared = {d for d in declared if not d.startswith("ac_match_t")}
+    assert {"ac_build", "ac_match", "ac_match_shard", "ac_free", "ac_compile"} <= declared
+    L = ac.lib()
+    for name in sorted(declared):
+        assert hasattr(L, name), name
+    assert set(ac.EXPORTED) == declared
+    assert "sm_100a" in ac.version()
+
+
+def test_status_strings():
+    L = ac.lib()
+    for s in range(8):
+        assert L.ac_status_string(s).decode().startswith("AC_")
+
+
+def _map_states(o: Oracle, t: ac.HostTable, forward: bool, pats):
+    """oracle state -> builder state, by walking each oracle state's string."""
+    C = t.info["n_classes"]
+    stride = t.info["row_stride"]
+    eb = t.info["entry_bytes"]
+    mask = 0x7FFF if eb == 2 else 0x7FFFFFFF
+    stt = t.stt.astype(np.int64)
+    strs = {0: b""}
+    frontier = [0]
+    while frontier:
+        nxt = []
+        for s in frontier:
+            for a in range(256):
+                u = o.goto(s, a)
+                if u is None or (s == 0 and u == 0):
+                    continue
+                strs[u] = strs[s] + bytes([a])
+                nxt.append(u)
+        frontier = nxt
+    mp = {}
+    for s, w in strs.items():
+        b = 0
+        for a in w:
+            b = int(stt[b, t.class_map[a]] & mask)
+        mp[s] = b
+    assert stride >= C
+    return mp, stt, mask
+
+
+def _check_builder(pats, forward: bool):
+    opats = pats if forward else [p[::-1] for p in pats]
+    o = Oracle(opats)
+    t = ac.compile_table(pats, forward=forward)
+    assert t.info["n_states"] == o.num_states
+    assert t.info["maxlen"] == max(len(p) for p in pats)
+    mp, stt, mask = _map_states(o, t, forward, pats)
+    assert sorted(mp.values()) == list(range(o.num_states))  # a bijection
+    flag = 0x8000 if t.info["entry_bytes"] == 2 else 0x80000000
+    # BFS numbering: depth is non-decreasing with the builder's state id
+    depth_by_b = {mp[s]: o.depth(s) for s in mp}
+    d = [depth_by_b[i] for i in range(o.num_states)]
+    assert d == sorted(d)
+    for s, b in mp.items():
+        outs = o.output(s)
+        assert t.out_ids[t.out_off[b]:t.out_off[b + 1]].tolist() == outs
+        row = stt[b]
+        for a in range(256):
+            u = o.delta(s, a)
+            e = int(row[t.class_map[a]])
+            assert e & mask == mp[u], (s, a)
+            assert bool(e & flag) == bool(o.output(u)), (s, a)
+
+
+def test_builder_worked_example_forward():
+    pats = [b"he", b"she", b"his", b"hers"]
+    _check_builder(pats, forward=True)
+    # P:66-68 through the builder, in creation-order names via the oracle map
+    o = Oracle(pats)
+    t = ac.compile_table(pats, forward=True)
+    mp, stt, mask = _map_states(o, t, True, pats)
+    inv = {v: k for k, v in mp.items()}
+    walk = []
+    s = 0
+    for ch in b"ushers":
+        s = int(stt[s, t.class_map[ch]] & mask)
+        walk.append(inv[s])
+    assert walk == [0, 3, 4, 5, 8, 9]
+
+
+@pytest.mark.parametrize("forward", [True, False])
+@pytest.mark.parametrize("seed", range(25))
+def test_builder_random_tiny(seed, forward):
+    rng = random.Random(seed)
+    A = rng.randint(1, 5)
+    alphabet = list(range(97, 97 + A)) if seed % 3 else [0, 255, 7, 128, 64][:A]
+    pats = [bytes(rng.choice(alphabet) for _ in range(rng.randint(1, 7))) for _ in range(rng.randint(1, 12))]
+    _check_builder(pats, forward)
+
+
+@pytest.mark.parametrize("forward", [True, False])
+def test_builder_c1_dictionary(forward):
+    import synth
+    _check_builder(synth.make("c1", n=1 << 12).patterns, forward)
+
+
+def test_builder_snort_like_entry4():
+    import synth
+    pats = synth.patterns_snort(150, 77)
+    t = ac.compile_table(pats, entry_bytes=4)
+    assert t.info["entry_bytes"] == 4 and t.info["row_stride"] % 2 == 1
+    _check_builder(pats, False)
+
+
+def test_classes_and_stride():
+    t = ac.compile_table([b"abc", b"zz"])
+    assert t.info["n_classes"] == 5  # a, b, c, z + class 0
+    assert t.class_map[ord("a")] == 1 and t.class_map[ord("z")] == 4 and t.class_map[0] == 0
+    words = t.info["row_stride"] * t.info["entry_bytes"] // 4
+    assert words % 2 == 1  # odd number of 4-byte words per row
+    all_bytes = [bytes([b]) for b in range(256)]
+    t2 = ac.compile_table(all_bytes)
+    assert t2.info["n_classes"] == 256 and list(t2.class_map) == list(range(256))
+
+
+def test_builder_errors():
+    with pytest.raises(ac.AcError) as e:
+        ac.compile_table([b"ok", b""])
+    assert e.value.status == ac.AC_ERR_EMPTY_PATTERN
+    rng = random.Random(3)
+    many = [bytes(rng.randrange(97, 123) for _ in range(8)) for _ in range(8000)]  # > 32768 states
+    with pytest.raises(ac.AcError) as e:
+        ac.compile_table(many, entry_bytes=2)
+    assert e.value.status == ac.AC_ERR_TOO_LARGE
+    with pytest.raises(ac.AcError):
+        ac.compile_table([b"a"], entry_bytes=3)
+
+
+def test_empty_dictionary_compiles():
+    t = ac.compile_table([])
+    assert t.info["n_states"] == 1 and t.info["out_entries"] == 0
+
+
+@pytest.mark.skipif(torch.cuda.is_available(), reason="checks the no-GPU failure mode")
+def test_no_device_fails_loudly():
+    with pytest.raises(ac.AcError) as e:
+        ac.build([b"he"], device=0)
+    assert e.value.status in (ac.AC_ERR_NO_DEVICE, ac.AC_ERR_CUDA)
