@@ -99,7 +99,11 @@ typedef struct {
     uint32_t hot_rows;     /* rows resident in shared memory                */
     uint32_t maxlen;       /* longest pattern                               */
     uint32_t forward;
-    uint32_t reserved;
+    uint32_t info_col;     /* entry index of each row's output summary: a u32
+                              payload (the pattern id when |output| == 1,
+                              else the CSR offset) followed by the count
+                              (u16 saturating at 0xFFFF if entry_bytes == 2,
+                              else u32)                                      */
     uint64_t stt_bytes;    /* S * row_stride * entry_bytes                  */
     uint64_t out_entries;  /* sum over states of |output(s)|                */
 } ac_stt_info;
@@ -119,6 +123,9 @@ typedef struct {
     uint32_t kernel;       /* AC_KERNEL_*                                    */
     uint32_t chain_bytes;  /* bytes owned per thread chain (0 = auto; STAGED:
                               rounded to the tile width)                     */
+    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..5 (DESIGN.md
+                              "Staged variants": threads x chains/thread x
+                              tile width x ring depth)                       */
     uint32_t n_events;     /* pairs available in `events`                    */
     void **events;         /* optional cudaEvent_t[2 * n_events]: events[2i]
                               and events[2i+1] are recorded on the stream
@@ -195,7 +202,8 @@ ac_status ac_match_host(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac
  * automaton.  ac_table_export copies any non-NULL array out:
  *   class_map[256]            byte -> class
  *   stt[S * row_stride]       entries of entry_bytes each: low bits = next
- *                             state, top bit (15 or 31) = output(next) != {}
+ *                             state, top bit (15 or 31) = output(next) != {};
+ *                             columns >= info_col hold the output summary
  *   out_off[S + 1], out_ids[out_entries]   output CSR, ids ascending
  */
 ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n_patterns,

@@ -59,12 +59,13 @@ class ac_stt_info(ctypes.Structure):
     _fields_ = [("n_patterns", ctypes.c_uint32), ("n_states", ctypes.c_uint32), ("n_classes", ctypes.c_uint32),
                 ("row_stride", ctypes.c_uint32), ("entry_bytes", ctypes.c_uint32), ("tier", ctypes.c_uint32),
                 ("hot_rows", ctypes.c_uint32), ("maxlen", ctypes.c_uint32), ("forward", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32), ("stt_bytes", ctypes.c_uint64), ("out_entries", ctypes.c_uint64)]
+                ("info_col", ctypes.c_uint32), ("stt_bytes", ctypes.c_uint64), ("out_entries", ctypes.c_uint64)]
 
 
 class ac_match_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("kernel", ctypes.c_uint32), ("chain_bytes", ctypes.c_uint32),
-                ("n_events", ctypes.c_uint32), ("events", ctypes.POINTER(ctypes.c_void_p))]
+                ("variant", ctypes.c_uint32), ("n_events", ctypes.c_uint32),
+                ("events", ctypes.POINTER(ctypes.c_void_p))]
 
 
 _lib = None
@@ -188,8 +189,8 @@ def _check_text(text: torch.Tensor):
         raise ValueError("text must be 1-D and contiguous")
 
 
-def _mopts(kernel: int, chain_bytes: int, events=None):
-    o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, 0, None)
+def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, events=None):
+    o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, 0, None)
     if events:
         arr = (ctypes.c_void_p * (2 * len(events)))(*[e.cuda_event for pair in events for e in pair])
         o.n_events = len(events)
@@ -200,10 +201,11 @@ def _mopts(kernel: int, chain_bytes: int, events=None):
 
 def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: torch.Tensor, *,
                 n_halo: int = 0, base: int = 0, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0,
-                events=None) -> int:
+                variant: int = 0, events=None) -> int:
     """Enqueue the scan; result (int64[2] CUDA) receives (count, status).
-    ``text`` holds n_owned + n_halo bytes.  ``events``: optional list of
-    (start, end) torch.cuda.Event pairs (already created, i.e. recorded
+    ``text`` holds n_owned + n_halo bytes.  ``kernel``/``chain_bytes``/
+    ``variant`` select the scan (ac_match_opts).  ``events``: optional list
+    of (start, end) torch.cuda.Event pairs (already created, i.e. recorded
     once) recorded around each kernel launch.  Returns the number of kernel
     launches issued."""
     _check_text(text)
@@ -220,32 +222,31 @@ def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: 
         cap = out.numel()
         # non-NULL selects list mode; with cap == 0 the status gates every write
         optr = out.data_ptr() if cap else result.data_ptr()
-    o = _mopts(kernel, chain_bytes, events)
+    o = _mopts(kernel, chain_bytes, variant, events)
     L = lib()
     _check(L.ac_match_async(stt.handle, text.data_ptr() if n_total else None, n_total - n_halo, n_halo, base,
                             optr, cap, result.data_ptr(), _stream_ptr(stream), ctypes.byref(o)))
     return int(L.ac_last_launch_count())
 
 
-def count(stt: Stt, text: torch.Tensor, *, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0) -> int:
-    """Number of occurrences (count-only scan)."""
+def count(stt: Stt, text: torch.Tensor, *, n_halo: int = 0, stream=None, **knobs) -> int:
+    """Number of occurrences (count-only scan); knobs as in match_async."""
     res = torch.zeros(2, dtype=torch.int64, device=text.device)
-    match_async(stt, text, None, res, stream=stream, kernel=kernel, chain_bytes=chain_bytes)
+    match_async(stt, text, None, res, n_halo=n_halo, stream=stream, **knobs)
     return int(res[0].item())
 
 
 def match(stt: Stt, text: torch.Tensor, out: torch.Tensor | None = None, *, n_halo: int = 0, base: int = 0,
-          stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0):
+          stream=None, **knobs):
     """Phase 2: (count, records) with records = out[:count] in canonical
     (start, pattern) order.  Without ``out`` a count pass sizes the buffer."""
     res = torch.zeros(2, dtype=torch.int64, device=text.device)
     if out is None:
-        match_async(stt, text, None, res, n_halo=n_halo, base=base, stream=stream, kernel=kernel,
-                    chain_bytes=chain_bytes)
+        match_async(stt, text, None, res, n_halo=n_halo, base=base, stream=stream, **knobs)
         need = int(res[0].item())
         out = torch.empty(max(1, need), dtype=torch.int64, device=text.device)
         res.zero_()
-    match_async(stt, text, out, res, n_halo=n_halo, base=base, stream=stream, kernel=kernel, chain_bytes=chain_bytes)
+    match_async(stt, text, out, res, n_halo=n_halo, base=base, stream=stream, **knobs)
     c, st = (int(x) for x in res.tolist())
     if st == AC_ERR_CAPACITY:
         raise CapacityError(st, f"{c} records do not fit in {out.numel()}", c)

@@ -33,7 +33,6 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
         if (e_ != cudaSuccess) return cuda_fail(e_, what); \
     } while (0)
 
-static const StagedConfig kStaged{256, 2, 64, 3};
 static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
 static const uint64_t kStagedMinBytes = 64 * 1024;
 static const uint64_t kStagedMinChain = 256;
@@ -86,22 +85,41 @@ static ac_status check_device(int device, cudaDeviceProp *prop) {
     return AC_OK;
 }
 
-static size_t staged_stt_budget(const ac_stt *h) {
-    size_t fixed = staged_smem_bytes(kStaged, 0) + 1024;  // + static smem / slack
+// Shared memory left for STT rows by a staged variant (v >= 1) or by the
+// global-only kernel (v == 0).
+static size_t stt_budget(const ac_stt *h, int v) {
+    const size_t fixed = (v ? staged_smem_bytes(staged_variant(v), 0) : 256) + 1024;  // + static smem / slack
     return h->smem_optin > fixed ? h->smem_optin - fixed : 0;
 }
 
-static SttView view_of(const ac_stt *h) {
-    SttView v;
-    v.stt = h->d_stt;
-    v.cmap = h->d_class_map;
-    v.out_off = h->d_out_off;
-    v.out_ids = h->d_out_ids;
-    v.stride = h->host.row_stride;
-    v.n_states = h->host.n_states;
-    v.smem_rows = h->tier == AC_TIER_GLOBAL ? 0 : h->hot_rows;
-    v.halo = h->host.maxlen ? h->host.maxlen - 1 : 0;
-    return v;
+static size_t row_bytes(const ac_stt *h) { return (size_t)h->host.row_stride * h->host.entry_bytes; }
+
+// STT view for one launch: the rows a kernel stages are capped by its budget.
+static SttView view_of(const ac_stt *h, int v) {
+    SttView s;
+    s.stt = h->d_stt;
+    s.cmap = h->d_class_map;
+    s.out_off = h->d_out_off;
+    s.out_ids = h->d_out_ids;
+    s.stride = h->host.row_stride;
+    s.n_states = h->host.n_states;
+    s.halo = h->host.maxlen ? h->host.maxlen - 1 : 0;
+    s.info_col = h->host.info_col;
+    uint64_t rows = h->tier == AC_TIER_GLOBAL ? 0 : h->hot_rows;
+    const uint64_t cap = stt_budget(h, v) / row_bytes(h);
+    s.smem_rows = (uint32_t)(rows < cap ? rows : cap);
+    return s;
+}
+
+static size_t smem_of(const ac_stt *h, const SttView &v) {
+    return ((size_t)v.smem_rows * row_bytes(h) + 15) / 16 * 16;
+}
+
+// The kernel's tier: SMEM only when every row is resident, GLOBAL when none.
+static uint32_t tier_of(const ac_stt *h, const SttView &v) {
+    if (v.smem_rows == 0) return AC_TIER_GLOBAL;
+    if (v.smem_rows >= h->host.n_states) return AC_TIER_SMEM;
+    return AC_TIER_HYBRID;
 }
 
 static void free_device(ac_stt *h) {
@@ -152,19 +170,32 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     AC_CUDA(cudaMemsetAsync(d_res, 0, sizeof(ac_result), stream), "memset result");
     if (n_owned == 0 || h->host.n_patterns == 0) return AC_OK;
 
-    const SttView st = view_of(h);
-    const size_t smem_stt = (size_t)st.smem_rows * st.stride * h->host.entry_bytes;
-    const size_t smem_stt16 = (smem_stt + 15) / 16 * 16;
-    const uint32_t eb = h->host.entry_bytes, tier = h->tier;
+    const uint32_t eb = h->host.entry_bytes;
     const uint64_t req_chain = opts ? opts->chain_bytes : 0;
     if (kernel == AC_KERNEL_AUTO) kernel = n_owned >= kStagedMinBytes ? AC_KERNEL_STAGED : AC_KERNEL_GLOBAL;
+    int variant = opts ? (int)opts->variant : 0;
+    if (variant < 0 || variant > staged_variant_count()) {
+        set_error("unknown staged variant");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (variant == 0) {
+        // SMEM tier: the deepest ring that still holds the whole table;
+        // otherwise the variant with the largest STT budget.
+        variant = 2;
+        const uint64_t need = (uint64_t)h->host.n_states * row_bytes(h);
+        if (h->tier == AC_TIER_SMEM && need <= stt_budget(h, 1)) variant = 1;
+    }
+    const SttView sg = view_of(h, 0), ss = view_of(h, variant);
+    const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
+    const size_t smem_g = smem_of(h, sg), smem_s = smem_of(h, ss);
+    const StagedConfig cfg = staged_variant(variant);
 
     // --- geometry: [head | main (staged) | tail] or a single global region
     Region ra{0, 0, kGlobalTailChain, 0, 0}, rb{0, 0, kGlobalTailChain, 0, 0};
     StagedGeom g{0, 0, 0, 0, 0};
     CUtensorMap tmap;
     if (kernel == AC_KERNEL_STAGED) {
-        const uint64_t W = (uint64_t)kStaged.width, R = (uint64_t)kStaged.threads * kStaged.k;
+        const uint64_t W = (uint64_t)cfg.width, R = (uint64_t)cfg.threads * cfg.k;
         uint64_t head = (16 - (reinterpret_cast<uintptr_t>(d_text) & 15)) & 15;
         if (head > n_owned) head = n_owned;
         const uint64_t avail = n_owned - head;
@@ -196,10 +227,12 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             cuuint64_t strides[1] = {(cuuint64_t)L};
             cuuint32_t box[2] = {(cuuint32_t)W, (cuuint32_t)(R < 256 ? R : 256)};
             cuuint32_t estr[2] = {1, 1};
+            const CUtensorMapSwizzle swz = W == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                           : W == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                     : CU_TENSOR_MAP_SWIZZLE_32B;
             CUresult cr = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, (void *)(d_text + head), dims, strides, box,
-                              estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                              W == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
-                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                              estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             if (cr != CUDA_SUCCESS) {
                 set_error("cuTensorMapEncodeTiled failed with CUresult " + std::to_string((int)cr));
                 return AC_ERR_CUDA;
@@ -220,29 +253,32 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     const uint64_t n_chains = ra.n_chains + g.n_chains + rb.n_chains;
     const bool any_global = ra.n_chains + rb.n_chains > 0;
 
-    // --- workspace: counts | chain_end | tile_state | counter
     ScanOut so{};
     so.base = base;
     so.res = d_res;
     so.out = reinterpret_cast<uint64_t *>(d_out);
-    void *ws = nullptr;
-    if (!emit) {
-        so.total = reinterpret_cast<unsigned long long *>(&d_res->count);
+    auto scan = [&](int mode, const char *gname, const char *sname) -> ac_status {
         if (any_global) {
             pre();
-            AC_CUDA(launch_scan_global(MODE_COUNT_TOTAL, eb, tier, d_text, n_total, st, ra, rb, so, smem_stt16, stream), "k_scan_global(count)");
-            post("k_scan_global(count)");
+            AC_CUDA(launch_scan_global(mode, eb, tier_g, d_text, n_total, sg, ra, rb, so, smem_g, stream), gname);
+            post(gname);
         }
         if (g.n_chains) {
             pre();
-            AC_CUDA(launch_scan_staged(MODE_COUNT_TOTAL, eb, tier, tmap, d_text + g.m0, st, g, kStaged, so, smem_stt16,
-                                       stream, nullptr), "k_scan_staged(count)");
-            post("k_scan_staged(count)");
+            AC_CUDA(launch_scan_staged(mode, eb, tier_s, variant, tmap, d_text + g.m0, ss, g, so, smem_s, stream),
+                    sname);
+            post(sname);
         }
         return AC_OK;
+    };
+    if (!emit) {
+        so.total = reinterpret_cast<unsigned long long *>(&d_res->count);
+        return scan(MODE_COUNT_TOTAL, "k_scan_global(count)", "k_scan_staged(count)");
     }
+    // --- list mode: counts | chain_end | tile_state | counter
     const size_t tiles = offsets_tiles(n_chains);
     const size_t bytes = n_chains * 8 * 2 + tiles * 8 + 16;
+    void *ws = nullptr;
     AC_CUDA(cudaMallocAsync(&ws, bytes, stream), "cudaMallocAsync(workspace)");
     uint64_t *counts = static_cast<uint64_t *>(ws);
     uint64_t *chain_end = counts + n_chains;
@@ -250,37 +286,16 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     unsigned int *counter = reinterpret_cast<unsigned int *>(tile_state + tiles);
     so.chain_counts = counts;
     so.chain_end = chain_end;
-    ac_status rc = AC_OK;
     auto run = [&]() -> ac_status {
         AC_CUDA(cudaMemsetAsync(tile_state, 0, tiles * 8 + 16, stream), "memset workspace");
-        if (any_global) {
-            pre();
-            AC_CUDA(launch_scan_global(MODE_COUNT_CHAINS, eb, tier, d_text, n_total, st, ra, rb, so, smem_stt16, stream), "k_scan_global(count)");
-            post("k_scan_global(count)");
-        }
-        if (g.n_chains) {
-            pre();
-            AC_CUDA(launch_scan_staged(MODE_COUNT_CHAINS, eb, tier, tmap, d_text + g.m0, st, g, kStaged, so, smem_stt16,
-                                       stream, nullptr), "k_scan_staged(count)");
-            post("k_scan_staged(count)");
-        }
+        ac_status rc = scan(MODE_COUNT_CHAINS, "k_scan_global(count)", "k_scan_staged(count)");
+        if (rc != AC_OK) return rc;
         pre();
         AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream), "k_offsets");
         post("k_offsets");
-        if (any_global) {
-            pre();
-            AC_CUDA(launch_scan_global(MODE_EMIT, eb, tier, d_text, n_total, st, ra, rb, so, smem_stt16, stream), "k_scan_global(emit)");
-            post("k_scan_global(emit)");
-        }
-        if (g.n_chains) {
-            pre();
-            AC_CUDA(launch_scan_staged(MODE_EMIT, eb, tier, tmap, d_text + g.m0, st, g, kStaged, so, smem_stt16, stream,
-                                       nullptr), "k_scan_staged(emit)");
-            post("k_scan_staged(emit)");
-        }
-        return AC_OK;
+        return scan(MODE_EMIT, "k_scan_global(emit)", "k_scan_staged(emit)");
     };
-    rc = run();
+    const ac_status rc = run();
     cudaFreeAsync(ws, stream);
     return rc;
 }
@@ -359,6 +374,7 @@ static void fill_info(const ac_table &t, ac_stt_info *info) {
     info->entry_bytes = t.entry_bytes;
     info->maxlen = t.maxlen;
     info->forward = t.forward;
+    info->info_col = t.info_col;
     info->stt_bytes = (uint64_t)t.n_states * t.row_stride * t.entry_bytes;
     info->out_entries = t.out_ids.size();
 }
@@ -425,7 +441,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     // residency tier
     const size_t row_bytes = (size_t)t.row_stride * t.entry_bytes;
     const size_t stt_bytes = (size_t)t.n_states * row_bytes;
-    const size_t budget = staged_stt_budget(h);
+    const size_t budget = stt_budget(h, 2);  // the largest staged budget
     uint32_t tier = opts ? opts->tier : AC_TIER_AUTO;
     uint32_t hot = opts ? opts->hot_rows : 0;
     if (tier == AC_TIER_AUTO) tier = stt_bytes <= budget ? AC_TIER_SMEM : AC_TIER_HYBRID;

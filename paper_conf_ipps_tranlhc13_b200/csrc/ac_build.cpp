@@ -152,17 +152,26 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
             set_error("entry_bytes=2 needs <= 32768 states");
             return AC_ERR_TOO_LARGE;
         }
-        // odd number of 4-byte words per row
-        uint32_t stride;
+        // Row = C transition entries, then the state's output summary (so a
+        // flagged transition learns |output(next)| and, when it is 1, the
+        // pattern id from the row it is about to walk anyway):
+        //   eb=2: entries [P, P+1] = u32 payload (P = C rounded to even), [P+2] = u16 count
+        //   eb=4: entry C = u32 payload, entry C+1 = u32 count
+        // payload = the pattern id if count == 1, else the CSR offset.
+        // The row is padded to an odd number of 4-byte words.
+        uint32_t stride, info_col;
         if (eb == 2) {
-            uint32_t words = (C + 1) / 2;
+            info_col = (C + 1) & ~1u;
+            uint32_t words = (info_col + 3 + 1) / 2;
             if (words % 2 == 0) words++;
             stride = words * 2;
         } else {
-            stride = C | 1u;
+            info_col = C;
+            stride = (C + 2) | 1u;
         }
         t.n_states = S;
         t.row_stride = stride;
+        t.info_col = info_col;
         t.entry_bytes = eb;
         t.stt.assign((size_t)S * stride * eb, 0);
         t.out_off.assign(S + 1, 0);
@@ -183,6 +192,17 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
         }
         for (uint32_t i = 0; i < S; i++) {
             const int32_t *row = &go[(size_t)order[i] * C];
+            const std::vector<uint32_t> &v = out[order[i]];
+            const uint32_t payload = v.size() == 1 ? v[0] : t.out_off[i];
+            uint8_t *r = &t.stt[(size_t)i * stride * eb];
+            std::memcpy(r + (size_t)info_col * eb, &payload, 4);
+            if (eb == 2) {
+                uint16_t c16 = (uint16_t)std::min<size_t>(v.size(), 0xFFFF);
+                std::memcpy(r + (size_t)(info_col + 2) * 2, &c16, 2);
+            } else {
+                uint32_t c32 = (uint32_t)v.size();
+                std::memcpy(r + (size_t)(info_col + 1) * 4, &c32, 4);
+            }
             for (uint32_t c = 0; c < C; c++) {
                 uint32_t nx = rank[(uint32_t)row[c]];
                 bool flag = !out[(uint32_t)row[c]].empty();

@@ -89,6 +89,32 @@ __device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uin
     return e & EntryBits<E>::MASK;
 }
 
+// Output summary of state s, stored in the padding of its own STT row
+// (builder: payload u32 at info_col, then the count), read through the same
+// residency tier as the transitions -- no dependent global CSR loads for the
+// common single-output case.
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t out_count(const E *s_stt, const SttView &st, uint32_t s) {
+    const uint32_t idx = s * st.stride + st.info_col + (sizeof(E) == 2 ? 2 : 1);
+    uint32_t c = stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, idx);
+    if (sizeof(E) == 2 && c == 0xFFFFu) c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);
+    return c;
+}
+
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t out_payload(const E *s_stt, const SttView &st, uint32_t s) {
+    const uint32_t idx = s * st.stride + st.info_col;  // 4-byte aligned by construction
+    const uint32_t *sp = reinterpret_cast<const uint32_t *>(s_stt + idx);
+    const uint32_t *gp = reinterpret_cast<const uint32_t *>(static_cast<const E *>(st.stt) + idx);
+    if constexpr (TIER == AC_TIER_SMEM) {
+        return *sp;
+    } else if constexpr (TIER == AC_TIER_GLOBAL) {
+        return __ldg(gp);
+    } else {
+        return *((s < st.smem_rows) ? sp : gp);
+    }
+}
+
 // One transition inside the owned chunk: count or emit output(s) at pos.
 template <typename E, int TIER, int MODE>
 __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp, uint32_t byte, uint64_t pos,
@@ -98,12 +124,17 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
     uint32_t e = stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
     s = e & EntryBits<E>::MASK;
     if ((e & EntryBits<E>::FLAG) && live) {
-        uint32_t a = __ldg(st.out_off + s), z = __ldg(st.out_off + s + 1);
+        const uint32_t c = out_count<E, TIER>(s_stt, st, s);
         if constexpr (MODE == MODE_EMIT) {
-            uint64_t key0 = (so.base + pos) << 24;
-            for (uint32_t j = z; j > a; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
+            const uint64_t key0 = (so.base + pos) << 24;
+            const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
+            if (c == 1) {
+                so.out[--wp] = key0 | p;
+            } else {
+                for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
+            }
         } else {
-            cnt += z - a;
+            cnt += c;
         }
     }
 }
@@ -437,55 +468,73 @@ cudaError_t launch_scan_global(int mode, uint32_t eb, uint32_t tier, const uint8
     return launch_global_e<uint32_t, MODE_EMIT>(tier, text, n_total, st, a, b, so, smem, stream);
 }
 
-// The staged kernel is instantiated for one shape; DESIGN.md records why.
-static constexpr int ST_T = 256, ST_K = 2, ST_W = 64, ST_NST = 3;
+// Staged kernel shapes (threads, chains per thread, tile width, ring depth).
+// Variant 0 is "auto"; the table index is ac_match_opts.variant.
+static const StagedConfig kVariants[] = {
+    {256, 2, 64, 3},  // 1: 512 chains, 96 KB ring (SMEM-tier default)
+    {256, 2, 32, 2},  // 2: 512 chains, 32 KB ring (largest STT budget)
+    {512, 2, 32, 2},  // 3: 1024 chains, 64 KB ring
+    {256, 4, 32, 2},  // 4: 1024 chains (4 per thread), 64 KB ring
+    {512, 1, 64, 2},  // 5: 512 chains, 64 KB ring, 1 chain per thread
+};
+
+int staged_variant_count() { return (int)(sizeof(kVariants) / sizeof(kVariants[0])); }
+const StagedConfig &staged_variant(int v) { return kVariants[v - 1]; }
 
 size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt) {
     return 1024 + (size_t)cfg.stages * cfg.threads * cfg.k * cfg.width + 128 + 256 + smem_stt;
 }
 
-template <typename E, int TIER, int MODE>
-static cudaError_t launch_staged_t(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
-                                   const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream,
-                                   int *ctas) {
-    auto kern = k_scan_staged<E, TIER, MODE, ST_T, ST_K, ST_W, ST_NST>;
-    StagedConfig cfg{ST_T, ST_K, ST_W, ST_NST};
+template <typename E, int TIER, int MODE, int T, int K, int W, int NST>
+static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
+                                   const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
+    auto kern = k_scan_staged<E, TIER, MODE, T, K, W, NST>;
+    const StagedConfig cfg{T, K, W, NST};
     const size_t smem = staged_smem_bytes(cfg, smem_stt);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    const uint64_t R = (uint64_t)ST_T * ST_K;
+    const uint64_t R = (uint64_t)T * K;
     const unsigned grid = (unsigned)((g.n_chains + R - 1) / R);
-    if (ctas) *ctas = (int)grid;
     if (grid == 0) return cudaSuccess;
-    kern<<<grid, ST_T, smem, stream>>>(tmap, mtext, st, g, so);
+    kern<<<grid, T, smem, stream>>>(tmap, mtext, st, g, so);
     return cudaGetLastError();
 }
 
+template <typename E, int TIER, int MODE>
+static cudaError_t launch_staged_t(int variant, const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
+                                   const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t s) {
+    switch (variant) {
+        case 1: return launch_staged_v<E, TIER, MODE, 256, 2, 64, 3>(tmap, mtext, st, g, so, smem_stt, s);
+        case 2: return launch_staged_v<E, TIER, MODE, 256, 2, 32, 2>(tmap, mtext, st, g, so, smem_stt, s);
+        case 3: return launch_staged_v<E, TIER, MODE, 512, 2, 32, 2>(tmap, mtext, st, g, so, smem_stt, s);
+        case 4: return launch_staged_v<E, TIER, MODE, 256, 4, 32, 2>(tmap, mtext, st, g, so, smem_stt, s);
+        case 5: return launch_staged_v<E, TIER, MODE, 512, 1, 64, 2>(tmap, mtext, st, g, so, smem_stt, s);
+    }
+    return cudaErrorInvalidValue;
+}
+
 template <typename E, int MODE>
-static cudaError_t launch_staged_e(uint32_t tier, const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
-                                   const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t s,
-                                   int *ctas) {
+static cudaError_t launch_staged_e(int variant, uint32_t tier, const CUtensorMap &tmap, const uint8_t *mtext,
+                                   const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
+                                   cudaStream_t s) {
     switch (tier) {
-        case AC_TIER_SMEM: return launch_staged_t<E, AC_TIER_SMEM, MODE>(tmap, mtext, st, g, so, smem_stt, s, ctas);
-        case AC_TIER_HYBRID: return launch_staged_t<E, AC_TIER_HYBRID, MODE>(tmap, mtext, st, g, so, smem_stt, s, ctas);
-        default: return launch_staged_t<E, AC_TIER_GLOBAL, MODE>(tmap, mtext, st, g, so, smem_stt, s, ctas);
+        case AC_TIER_SMEM: return launch_staged_t<E, AC_TIER_SMEM, MODE>(variant, tmap, mtext, st, g, so, smem_stt, s);
+        case AC_TIER_HYBRID: return launch_staged_t<E, AC_TIER_HYBRID, MODE>(variant, tmap, mtext, st, g, so, smem_stt, s);
+        default: return launch_staged_t<E, AC_TIER_GLOBAL, MODE>(variant, tmap, mtext, st, g, so, smem_stt, s);
     }
 }
 
-cudaError_t launch_scan_staged(int mode, uint32_t eb, uint32_t tier, const CUtensorMap &tmap,
-                               const uint8_t *mtext, const SttView &st, const StagedGeom &g,
-                               const StagedConfig &cfg, const ScanOut &so, size_t smem_stt,
-                               cudaStream_t stream, int *ctas) {
-    if (cfg.threads != ST_T || cfg.k != ST_K || cfg.width != ST_W || cfg.stages != ST_NST)
-        return cudaErrorInvalidValue;
+cudaError_t launch_scan_staged(int mode, uint32_t eb, uint32_t tier, int variant, const CUtensorMap &tmap,
+                               const uint8_t *mtext, const SttView &st, const StagedGeom &g, const ScanOut &so,
+                               size_t smem_stt, cudaStream_t stream) {
     if (eb == 2) {
-        if (mode == MODE_COUNT_TOTAL) return launch_staged_e<uint16_t, MODE_COUNT_TOTAL>(tier, tmap, mtext, st, g, so, smem_stt, stream, ctas);
-        if (mode == MODE_COUNT_CHAINS) return launch_staged_e<uint16_t, MODE_COUNT_CHAINS>(tier, tmap, mtext, st, g, so, smem_stt, stream, ctas);
-        return launch_staged_e<uint16_t, MODE_EMIT>(tier, tmap, mtext, st, g, so, smem_stt, stream, ctas);
+        if (mode == MODE_COUNT_TOTAL) return launch_staged_e<uint16_t, MODE_COUNT_TOTAL>(variant, tier, tmap, mtext, st, g, so, smem_stt, stream);
+        if (mode == MODE_COUNT_CHAINS) return launch_staged_e<uint16_t, MODE_COUNT_CHAINS>(variant, tier, tmap, mtext, st, g, so, smem_stt, stream);
+        return launch_staged_e<uint16_t, MODE_EMIT>(variant, tier, tmap, mtext, st, g, so, smem_stt, stream);
     }
-    if (mode == MODE_COUNT_TOTAL) return launch_staged_e<uint32_t, MODE_COUNT_TOTAL>(tier, tmap, mtext, st, g, so, smem_stt, stream, ctas);
-    if (mode == MODE_COUNT_CHAINS) return launch_staged_e<uint32_t, MODE_COUNT_CHAINS>(tier, tmap, mtext, st, g, so, smem_stt, stream, ctas);
-    return launch_staged_e<uint32_t, MODE_EMIT>(tier, tmap, mtext, st, g, so, smem_stt, stream, ctas);
+    if (mode == MODE_COUNT_TOTAL) return launch_staged_e<uint32_t, MODE_COUNT_TOTAL>(variant, tier, tmap, mtext, st, g, so, smem_stt, stream);
+    if (mode == MODE_COUNT_CHAINS) return launch_staged_e<uint32_t, MODE_COUNT_CHAINS>(variant, tier, tmap, mtext, st, g, so, smem_stt, stream);
+    return launch_staged_e<uint32_t, MODE_EMIT>(variant, tier, tmap, mtext, st, g, so, smem_stt, stream);
 }
 
 cudaError_t launch_offsets(const uint64_t *counts, uint64_t n, uint64_t *chain_end, uint64_t *tile_state,

@@ -22,6 +22,7 @@ struct SttView {
     uint32_t n_states;
     uint32_t smem_rows;       // rows staged into shared memory
     uint32_t halo;            // maxlen - 1
+    uint32_t info_col;        // entry index of the row's output summary (payload u32, count)
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.
@@ -62,15 +63,16 @@ struct StagedConfig {
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,
                                uint64_t n_total, const SttView &st, const Region &a, const Region &b,
                                const ScanOut &so, size_t smem_bytes, cudaStream_t stream);
-cudaError_t launch_scan_staged(int mode, uint32_t entry_bytes, uint32_t tier, const CUtensorMap &tmap,
-                               const uint8_t *main_text, const SttView &st, const StagedGeom &g,
-                               const StagedConfig &cfg, const ScanOut &so, size_t smem_stt_bytes,
-                               cudaStream_t stream, int *ctas_out);
+cudaError_t launch_scan_staged(int mode, uint32_t entry_bytes, uint32_t tier, int variant, const CUtensorMap &tmap,
+                               const uint8_t *main_text, const SttView &st, const StagedGeom &g, const ScanOut &so,
+                               size_t smem_stt_bytes, cudaStream_t stream);
 cudaError_t launch_offsets(const uint64_t *counts, uint64_t n, uint64_t *chain_end, uint64_t *tile_state,
                            unsigned int *tile_counter, ac_result *res, uint64_t cap, int emitting,
                            cudaStream_t stream);
 
 size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
+int staged_variant_count();
+const StagedConfig &staged_variant(int v);  // v in [1, staged_variant_count()]
 size_t offsets_tiles(uint64_t n);
 
 }  // namespace acx

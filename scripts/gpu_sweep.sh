@@ -1,0 +1,7 @@
+#!/bin/bash
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 900 python -m pytest tests -m gpu -x -q -k "not slow" > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
+for c in c2 c1 c3 c4; do
+  timeout 600 python scripts/sweep.py --config $c --global-kernel --tiers auto,global > gpurun_out/sweep_$c.jsonl 2> gpurun_out/sweep_$c.err
+done

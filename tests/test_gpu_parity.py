@@ -38,7 +38,7 @@ def oracle_keys(o: Oracle, text, lo=None, hi=None) -> np.ndarray:
 def gpu_keys(stt, text_np: np.ndarray, **kw) -> np.ndarray:
     t = torch.from_numpy(np.ascontiguousarray(text_np)).cuda() if text_np.size else torch.empty(0, dtype=torch.uint8, device="cuda")
     c, recs = ac.match(stt, t, **kw)
-    cnt = ac.count(stt, t, **{k: v for k, v in kw.items() if k in ("kernel", "chain_bytes")})
+    cnt = ac.count(stt, t, **{k: v for k, v in kw.items() if k in ("kernel", "chain_bytes", "variant")})
     assert cnt == c
     return recs.cpu().numpy()
 
@@ -103,6 +103,17 @@ def test_c3_hybrid_and_global_tiers():
     for tier in (ac.TIER_AUTO, ac.TIER_GLOBAL):
         stt = ac.build(w.patterns, tier=tier)
         assert_same(gpu_keys(stt, w.text), want)
+
+
+@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5])
+@pytest.mark.parametrize("name", ["c1", "c2"])
+def test_staged_variants(variant, name):
+    w = synth.make(name, n=(2 << 20) + 4321, n_patterns=None if name == "c1" else 400)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    want = oracle_keys(o, w.text)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant, chain_bytes=96), want)
 
 
 @pytest.mark.parametrize("chain", [64, 128, 320, 1024, 4096, 65536])

@@ -84,9 +84,18 @@ def _check_builder(pats, forward: bool):
     depth_by_b = {mp[s]: o.depth(s) for s in mp}
     d = [depth_by_b[i] for i in range(o.num_states)]
     assert d == sorted(d)
+    ic = t.info["info_col"]
+    eb = t.info["entry_bytes"]
+    assert ic >= t.info["n_classes"] and (eb == 4 or ic % 2 == 0)
+    raw = t.stt.view(np.uint8).reshape(o.num_states, -1)
     for s, b in mp.items():
         outs = o.output(s)
         assert t.out_ids[t.out_off[b]:t.out_off[b + 1]].tolist() == outs
+        # output summary in the row padding: payload u32, then the count
+        payload = int(raw[b, ic * eb: ic * eb + 4].view(np.uint32)[0])
+        cnt = int(stt[b, ic + (2 if eb == 2 else 1)])
+        assert cnt == min(len(outs), 0xFFFF if eb == 2 else 1 << 32)
+        assert payload == (outs[0] if len(outs) == 1 else int(t.out_off[b]))
         row = stt[b]
         for a in range(256):
             u = o.delta(s, a)
