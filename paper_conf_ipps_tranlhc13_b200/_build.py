@@ -1,12 +1,15 @@
 """Builds libac.so in-tree with nvcc for sm_100a (no JIT, no torch extension).
 
-The built library lives next to this file so it travels with the repository
-snapshot to the GPU box.  Rebuilds only when a source is newer than the .so.
+Each translation unit is compiled to an object in parallel (the per-tier
+kernel instantiations dominate), then linked into one shared library that
+lives next to this file so it travels with the repository snapshot to the
+GPU box.  Rebuilds only when a source is newer than the .so.
 """
 from __future__ import annotations
 
 import os
 import subprocess
+from concurrent.futures import ThreadPoolExecutor
 from pathlib import Path
 
 PKG = Path(__file__).resolve().parent
@@ -14,13 +17,10 @@ ROOT = PKG.parent
 CSRC = PKG / "csrc"
 LIB = PKG / "libac.so"
 INCLUDE = ROOT / "include"
+OBJ = ROOT / "build" / "obj"
 
-NVCC_FLAGS = [
-    "-std=c++17", "-O3", "-lineinfo",
-    "-gencode", "arch=compute_100a,code=sm_100a",
-    "-Xcompiler", "-fPIC,-O2", "-shared",
-    "--expt-relaxed-constexpr",
-]
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+CFLAGS = ["-std=c++17", "-O3", "-lineinfo", *ARCH, "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr"]
 
 
 def sources() -> list[Path]:
@@ -36,8 +36,8 @@ def _stale() -> bool:
 
 
 def nvcc() -> str:
-    for c in (os.environ.get("NVCC"), "/usr/local/cuda/bin/nvcc", "nvcc"):
-        if c and (c == "nvcc" or Path(c).exists()):
+    for c in (os.environ.get("NVCC"), "/usr/local/cuda/bin/nvcc"):
+        if c and Path(c).exists():
             return c
     return "nvcc"
 
@@ -45,12 +45,21 @@ def nvcc() -> str:
 def build(force: bool = False, verbose: bool = False) -> Path:
     if not force and not _stale():
         return LIB
+    OBJ.mkdir(parents=True, exist_ok=True)
+    extra = ["-Xptxas=-v"] if verbose else []
+
+    def compile_one(src: Path) -> Path:
+        obj = OBJ / (src.name + ".o")
+        cmd = [nvcc(), *CFLAGS, *extra, f"-I{INCLUDE}", f"-I{CSRC}", "-c", str(src), "-o", str(obj)]
+        if verbose:
+            print(" ".join(cmd), flush=True)
+        subprocess.check_call(cmd)
+        return obj
+
+    with ThreadPoolExecutor(max_workers=max(1, min(8, os.cpu_count() or 1))) as ex:
+        objs = list(ex.map(compile_one, sources()))
     tmp = LIB.with_suffix(f".so.tmp{os.getpid()}")
-    cmd = [nvcc(), *NVCC_FLAGS, f"-I{INCLUDE}", f"-I{CSRC}", "-o", str(tmp), *map(str, sources())]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
+    subprocess.check_call([nvcc(), *ARCH, "-shared", "-o", str(tmp), *map(str, objs)])
     os.replace(tmp, LIB)
     return LIB
 

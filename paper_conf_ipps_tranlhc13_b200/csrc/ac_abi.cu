@@ -33,7 +33,8 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
         if (e_ != cudaSuccess) return cuda_fail(e_, what); \
     } while (0)
 
-static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
+static const uint64_t kGlobalTailChain = 64;
+static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)  // head/tail chains of the staged path
 static const uint64_t kStagedMinBytes = 64 * 1024;
 static const uint64_t kStagedMinChain = 256;
 
@@ -178,13 +179,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         set_error("unknown staged variant");
         return AC_ERR_INVALID_ARG;
     }
-    if (variant == 0) {
-        // SMEM tier: the deepest ring that still holds the whole table;
-        // otherwise the variant with the largest STT budget.
-        variant = 2;
-        const uint64_t need = (uint64_t)h->host.n_states * row_bytes(h);
-        if (h->tier == AC_TIER_SMEM && need <= stt_budget(h, 1)) variant = 1;
-    }
+    if (variant == 0) variant = kAutoVariant;
     const SttView sg = view_of(h, 0), ss = view_of(h, variant);
     const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
     const size_t smem_g = smem_of(h, sg), smem_s = smem_of(h, ss);
@@ -195,7 +190,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     StagedGeom g{0, 0, 0, 0, 0};
     CUtensorMap tmap;
     if (kernel == AC_KERNEL_STAGED) {
-        const uint64_t W = (uint64_t)cfg.width, R = (uint64_t)cfg.threads * cfg.k;
+        const uint64_t W = (uint64_t)cfg.width, R = (uint64_t)cfg.warps * 32 * cfg.k;
         uint64_t head = (16 - (reinterpret_cast<uintptr_t>(d_text) & 15)) & 15;
         if (head > n_owned) head = n_owned;
         const uint64_t avail = n_owned - head;
@@ -225,11 +220,12 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             }
             cuuint64_t dims[2] = {(cuuint64_t)L, (cuuint64_t)n_main};
             cuuint64_t strides[1] = {(cuuint64_t)L};
-            cuuint32_t box[2] = {(cuuint32_t)W, (cuuint32_t)(R < 256 ? R : 256)};
+            cuuint32_t box[2] = {(cuuint32_t)W, (cuuint32_t)(32 * cfg.k)};
             cuuint32_t estr[2] = {1, 1};
             const CUtensorMapSwizzle swz = W == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
                                            : W == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
-                                                     : CU_TENSOR_MAP_SWIZZLE_32B;
+                                           : W == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                                     : CU_TENSOR_MAP_SWIZZLE_NONE;
             CUresult cr = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, (void *)(d_text + head), dims, strides, box,
                               estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -441,7 +437,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     // residency tier
     const size_t row_bytes = (size_t)t.row_stride * t.entry_bytes;
     const size_t stt_bytes = (size_t)t.n_states * row_bytes;
-    const size_t budget = stt_budget(h, 2);  // the largest staged budget
+    const size_t budget = stt_budget(h, 1);  // a 48 KB-ring staged variant
     uint32_t tier = opts ? opts->tier : AC_TIER_AUTO;
     uint32_t hot = opts ? opts->hot_rows : 0;
     if (tier == AC_TIER_AUTO) tier = stt_bytes <= budget ? AC_TIER_SMEM : AC_TIER_HYBRID;

@@ -1,0 +1,471 @@
+// ac_kernels.cuh -- device code of the Aho-Corasick scan for sm_100a
+// (templates; instantiated once per STT tier in ac_tier_*.cu).
+//
+// The hot loop is the DFA walk of P:60-70: one dependent STT gather per text
+// byte (state <- delta(state, text[i]), O(n) transitions), with the
+// output function consulted when the entry's match flag (the paper's column
+// M) is set.  Text decomposition follows the paper's chunking: each
+// thread walks its own chunk, extended by the longest pattern so straddling
+// matches are found, with ownership by START position so every
+// occurrence is reported once (reading R9).  Because the automaton is built
+// over reversed patterns, every chain walks right to left: the (maxlen - 1)
+// halo to the right of the chunk is consumed first as a warm-up (no output)
+// and the chunk's matches then come out in descending (start, pattern) order,
+// which the emitter writes backwards from the chain's end offset -- the list
+// is canonical without any sort.
+//
+// Kernels:
+//   k_scan_staged  the paper's "shared memory approach" rebuilt
+//                  for sm_100a.  Each WARP owns 32*K chains of L bytes and a
+//                  private ring of NST shared-memory slots; one lane streams
+//                  the warp's text with 2-D TMA boxes (W bytes x 32*K chains,
+//                  plus one box of the next chains' first bytes for the
+//                  halo), each slot guarded by its own mbarrier.  Warps never
+//                  wait for each other (the only CTA barrier is after the STT
+//                  is staged), so the irregular gather latency of one warp
+//                  does not stall the SM.  The TMA swizzle (32B/64B) is the
+//                  hardware form of the paper's diagonal, bank-conflict-free
+//                  store: lane l reads its chain 16 B at a time
+//                  with conflict-free LDS.128.
+//   k_scan_global  the paper's "global memory only approach":
+//                  each thread reads its chain straight from global memory
+//                  (16-byte vector loads, L1-cached).  Also covers the
+//                  unaligned head and the ragged tail of the staged path.
+//
+// STT tiers: SMEM (whole table staged once per CTA),
+// HYBRID (BFS-prefix rows in shared memory, the rest through L1/L2 with a
+// generic load), GLOBAL (L1/L2 only).
+#pragma once
+
+#include "ac_scan.cuh"
+
+namespace acx {
+
+static constexpr int GT = 256;  // k_scan_global block size
+
+template <typename E>
+struct EntryBits;
+template <>
+struct EntryBits<uint16_t> {
+    static constexpr uint32_t FLAG = 0x8000u, MASK = 0x7fffu;
+};
+template <>
+struct EntryBits<uint32_t> {
+    static constexpr uint32_t FLAG = 0x80000000u, MASK = 0x7fffffffu;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// ------------------------------------------------------------------ tables
+template <typename E>
+__device__ __forceinline__ void stage_tables(uint8_t *s_cmap, E *s_stt, const SttView &st) {
+    const uint4 *c4 = reinterpret_cast<const uint4 *>(st.cmap);
+    uint4 *d4 = reinterpret_cast<uint4 *>(s_cmap);
+    for (int i = threadIdx.x; i < 16; i += blockDim.x) d4[i] = __ldg(c4 + i);
+    const size_t words = ((size_t)st.smem_rows * st.stride * sizeof(E) + 15) / 16;
+    const uint4 *src = reinterpret_cast<const uint4 *>(st.stt);
+    uint4 *dst = reinterpret_cast<uint4 *>(s_stt);
+    for (size_t i = threadIdx.x; i < words; i += blockDim.x) dst[i] = __ldg(src + i);
+}
+
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uint32_t hot, uint32_t s,
+                                             uint32_t idx) {
+    if constexpr (TIER == AC_TIER_SMEM) {
+        return s_stt[idx];
+    } else if constexpr (TIER == AC_TIER_GLOBAL) {
+        return __ldg(g_stt + idx);
+    } else {
+        const E *p = (s < hot) ? (s_stt + idx) : (g_stt + idx);
+        return *p;
+    }
+}
+
+// One transition with no output (halo warm-up).
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uint8_t *s_cmap, const E *s_stt,
+                                            const SttView &st) {
+    const uint32_t cls = s_cmap[byte];
+    const uint32_t e =
+        stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
+    return e & EntryBits<E>::MASK;
+}
+
+// Output summary of state s, stored in the padding of its own STT row
+// (builder: payload u32 at info_col, then the count), read through the same
+// residency tier as the transitions -- no dependent global CSR loads for the
+// common single-output case.
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t out_count(const E *s_stt, const SttView &st, uint32_t s) {
+    const uint32_t idx = s * st.stride + st.info_col + (sizeof(E) == 2 ? 2 : 1);
+    uint32_t c = stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, idx);
+    if (sizeof(E) == 2 && c == 0xFFFFu) c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);
+    return c;
+}
+
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t out_payload(const E *s_stt, const SttView &st, uint32_t s) {
+    const uint32_t idx = s * st.stride + st.info_col;  // 4-byte aligned by construction
+    const uint32_t *sp = reinterpret_cast<const uint32_t *>(s_stt + idx);
+    const uint32_t *gp = reinterpret_cast<const uint32_t *>(static_cast<const E *>(st.stt) + idx);
+    if constexpr (TIER == AC_TIER_SMEM) {
+        return *sp;
+    } else if constexpr (TIER == AC_TIER_GLOBAL) {
+        return __ldg(gp);
+    } else {
+        return *((s < st.smem_rows) ? sp : gp);
+    }
+}
+
+// One transition inside the owned chunk: count or emit output(s) at pos.
+template <typename E, int TIER, int MODE>
+__device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp, uint32_t byte, uint64_t pos,
+                                        bool live, const uint8_t *s_cmap, const E *s_stt, const SttView &st,
+                                        const ScanOut &so) {
+    const uint32_t cls = s_cmap[byte];
+    const uint32_t e =
+        stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
+    s = e & EntryBits<E>::MASK;
+    if ((e & EntryBits<E>::FLAG) && live) {
+        const uint32_t c = out_count<E, TIER>(s_stt, st, s);
+        if constexpr (MODE == MODE_EMIT) {
+            const uint64_t key0 = (so.base + pos) << 24;
+            const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
+            if (c == 1) {
+                so.out[--wp] = key0 | p;
+            } else {
+                for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
+            }
+        } else {
+            cnt += c;
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t byte_of(const uint4 &v, int bb) {
+    const uint32_t w = (bb >> 2) == 0 ? v.x : (bb >> 2) == 1 ? v.y : (bb >> 2) == 2 ? v.z : v.w;
+    return (w >> (8 * (bb & 3))) & 0xffu;
+}
+
+__device__ __forceinline__ unsigned long long warp_sum(unsigned long long v) {
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// ------------------------------------------------------- k_scan_global (K1)
+// Walk text[a, b) right to left; OWNED selects emission (else warm-up).
+template <typename E, int TIER, int MODE, bool OWNED>
+__device__ __forceinline__ void walk_global(const uint8_t *__restrict__ text, uint64_t a, uint64_t b, uint32_t &s,
+                                            uint64_t &cnt, uint64_t &wp, const uint8_t *s_cmap, const E *s_stt,
+                                            const SttView &st, const ScanOut &so) {
+    auto one = [&](uint32_t byte, uint64_t pos) {
+        if constexpr (OWNED)
+            ac_step<E, TIER, MODE>(s, cnt, wp, byte, pos, true, s_cmap, s_stt, st, so);
+        else
+            s = ac_move<E, TIER>(s, byte, s_cmap, s_stt, st);
+    };
+    uint64_t i = b;
+    while (i > a && (reinterpret_cast<uintptr_t>(text + i) & 15u)) {
+        --i;
+        one(__ldg(text + i), i);
+    }
+    while (i >= a + 16) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4 *>(text + i - 16));
+#pragma unroll
+        for (int bb = 15; bb >= 0; --bb) one(byte_of(v, bb), i - 16 + bb);
+        i -= 16;
+    }
+    while (i > a) {
+        --i;
+        one(__ldg(text + i), i);
+    }
+}
+
+template <typename E, int TIER, int MODE>
+__global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ text, uint64_t n_total, SttView st,
+                                                    Region ra, Region rb, ScanOut so) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint8_t *s_cmap = smem;
+    E *s_stt = reinterpret_cast<E *>(smem + 256);
+    stage_tables<E>(s_cmap, s_stt, st);
+    __syncthreads();
+    if constexpr (MODE == MODE_EMIT) {
+        if (so.res->status != AC_OK) return;  // capacity exceeded: write nothing
+    }
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool in_a = t < ra.n_chains;
+    const uint64_t ci = in_a ? t : t - ra.n_chains;
+    const uint64_t r_lo = in_a ? ra.lo : rb.lo, r_hi = in_a ? ra.hi : rb.hi;
+    const uint64_t r_len = in_a ? ra.chain_len : rb.chain_len, r_n = in_a ? ra.n_chains : rb.n_chains;
+    const uint64_t r_c0 = in_a ? ra.chain0 : rb.chain0;
+    uint64_t cnt = 0;
+    if (ci < r_n) {
+        const uint64_t lo = r_lo + ci * r_len;
+        const uint64_t own_hi = min(lo + r_len, r_hi);
+        const uint64_t walk_hi = min(own_hi + (uint64_t)st.halo, n_total);
+        const uint64_t g = r_c0 + ci;
+        uint64_t wp = 0;
+        if constexpr (MODE == MODE_EMIT) wp = so.chain_end[g];
+        uint32_t s = 0;
+        walk_global<E, TIER, MODE, false>(text, own_hi, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
+        walk_global<E, TIER, MODE, true>(text, lo, own_hi, s, cnt, wp, s_cmap, s_stt, st, so);
+        if constexpr (MODE == MODE_COUNT_CHAINS) so.chain_counts[g] = cnt;
+    }
+    if constexpr (MODE == MODE_COUNT_TOTAL) {
+        const unsigned long long tot = warp_sum(cnt);
+        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(so.total, tot);
+    }
+}
+
+// --------------------------------------------------------- TMA / mbarrier
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    uint32_t done;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
+        "[%4];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
+        : "memory");
+}
+
+// ------------------------------------------- k_scan_staged (warp-private TMA)
+template <int WARPS, int K, int W, int NST>
+struct StagedShape {
+    static constexpr int ROWS = 32 * K;               // chains per warp = TMA box rows (<= 256)
+    static constexpr int SLOT = ROWS * W;             // bytes per ring slot
+    static constexpr int WARP_RING = NST * SLOT;
+    static constexpr int RING = WARPS * WARP_RING;
+    static constexpr int BARS = (WARPS * NST * 8 + 15) / 16 * 16;
+    static constexpr uint32_t SWZ = W == 128 ? 7u : W == 64 ? 3u : W == 32 ? 1u : 0u;
+    static_assert(ROWS <= 256, "TMA box rows");
+    static_assert(W == 16 || W == 32 || W == 64 || W == 128, "tile width");
+    static_assert(SLOT % 512 == 0 || W == 16, "slots must keep the swizzle atom aligned");
+};
+
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST>
+__global__ void __launch_bounds__(WARPS * 32, 1)
+    k_scan_staged(const __grid_constant__ CUtensorMap tmap, const uint8_t *__restrict__ mtext, SttView st,
+                  StagedGeom g, ScanOut so) {
+    using Sh = StagedShape<WARPS, K, W, NST>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *ring = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ring + Sh::RING);
+    uint8_t *s_cmap = ring + Sh::RING + Sh::BARS;
+    E *s_stt = reinterpret_cast<E *>(s_cmap + 256);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    if (threadIdx.x < WARPS * NST) mbar_init(&bars[threadIdx.x], 1);
+    if (threadIdx.x == 0) {
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
+    }
+    stage_tables<E>(s_cmap, s_stt, st);
+    __syncthreads();  // the only CTA-wide barrier: tables staged, barriers initialised
+    if constexpr (MODE == MODE_EMIT) {
+        if (so.res->status != AC_OK) return;  // capacity exceeded: write nothing
+    }
+    const uint64_t row0 = (uint64_t)blockIdx.x * (WARPS * Sh::ROWS) + (uint64_t)warp * Sh::ROWS;
+    if (row0 >= g.n_chains) return;  // idle warp (no later CTA barrier)
+
+    uint8_t *wring = ring + warp * Sh::WARP_RING;
+    uint64_t *wbar = bars + warp * NST;
+    const uint64_t L = g.chain_len;
+    const uint32_t H = st.halo;
+    const uint32_t nh0 = (H + W - 1) / W;
+    const bool tma_halo = (uint64_t)nh0 * W <= L;  // the halo window lies inside the next chain
+    const uint32_t nh = tma_halo ? nh0 : 0;
+    const uint32_t m = nh + (uint32_t)(L / W);
+
+    auto issue = [&](uint32_t j) {
+        const uint32_t slot = j % NST;
+        int x, y;
+        if (j < nh) {  // halo: first bytes of the next chains (the row below)
+            x = (int)((nh - 1 - j) * W);
+            y = (int)(row0 + 1);
+        } else {
+            x = (int)(L - (uint64_t)(j - nh + 1) * W);
+            y = (int)row0;
+        }
+        mbar_expect_tx(&wbar[slot], Sh::SLOT);
+        tma_load_2d(wring + slot * Sh::SLOT, &tmap, x, y, &wbar[slot]);
+    };
+    if (lane == 0)
+        for (uint32_t j = 0; j < (uint32_t)NST && j < m; j++) issue(j);
+
+    uint32_t s[K], hlen[K];
+    uint64_t cnt[K], wp[K], cbase[K];
+    bool live[K];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const uint64_t c = row0 + k * 32 + lane;
+        live[k] = c < g.n_chains;
+        s[k] = 0;
+        cnt[k] = 0;
+        wp[k] = 0;
+        cbase[k] = c * L;  // main-region offset of the chain's first byte
+        const uint64_t rest = live[k] ? g.n_readable - (c + 1) * L : 0;
+        hlen[k] = (uint32_t)(rest < H ? rest : H);
+        if constexpr (MODE == MODE_EMIT)
+            if (live[k]) wp[k] = so.chain_end[g.chain0 + c];
+        // the last chain's halo row is outside the tensor map (and any halo
+        // wider than the next chain): warm up from global memory instead
+        if (live[k] && (!tma_halo || c + 1 == g.n_chains)) {
+            for (int h = (int)hlen[k] - 1; h >= 0; --h)
+                s[k] = ac_move<E, TIER>(s[k], __ldg(mtext + cbase[k] + L + h), s_cmap, s_stt, st);
+            hlen[k] = 0;
+        }
+    }
+
+    for (uint32_t j = 0; j < m; j++) {
+        const uint32_t slot = j % NST;
+        mbar_wait(&wbar[slot], (j / NST) & 1u);
+        const uint8_t *tile = wring + slot * Sh::SLOT;
+        if (j < nh) {
+            const uint32_t col0 = (nh - 1 - j) * W;  // offset inside the halo window
+#pragma unroll
+            for (int q = W / 16 - 1; q >= 0; --q) {
+                uint4 v[K];
+#pragma unroll
+                for (int k = 0; k < K; k++) {
+                    const uint32_t logical = (k * 32 + lane) * W + q * 16;
+                    v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
+                }
+#pragma unroll
+                for (int bb = 15; bb >= 0; --bb) {
+#pragma unroll
+                    for (int k = 0; k < K; k++)
+                        if (col0 + q * 16 + bb < hlen[k])
+                            s[k] = ac_move<E, TIER>(s[k], byte_of(v[k], bb), s_cmap, s_stt, st);
+                }
+            }
+        } else {
+            const uint64_t col0 = L - (uint64_t)(j - nh + 1) * W;
+#pragma unroll
+            for (int q = W / 16 - 1; q >= 0; --q) {
+                uint4 v[K];
+#pragma unroll
+                for (int k = 0; k < K; k++) {
+                    const uint32_t logical = (k * 32 + lane) * W + q * 16;
+                    v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
+                }
+#pragma unroll
+                for (int bb = 15; bb >= 0; --bb) {
+#pragma unroll
+                    for (int k = 0; k < K; k++) {
+                        const uint64_t pos = g.m0 + cbase[k] + col0 + q * 16 + bb;
+                        ac_step<E, TIER, MODE>(s[k], cnt[k], wp[k], byte_of(v[k], bb), pos, live[k], s_cmap, s_stt,
+                                               st, so);
+                    }
+                }
+            }
+        }
+        __syncwarp();  // every lane is done with this slot
+        if (lane == 0 && j + NST < m) issue(j + NST);
+    }
+
+    if constexpr (MODE == MODE_COUNT_CHAINS) {
+#pragma unroll
+        for (int k = 0; k < K; k++)
+            if (live[k]) so.chain_counts[g.chain0 + row0 + k * 32 + lane] = cnt[k];
+    }
+    if constexpr (MODE == MODE_COUNT_TOTAL) {
+        unsigned long long sum = 0;
+#pragma unroll
+        for (int k = 0; k < K; k++) sum += cnt[k];
+        sum = warp_sum(sum);
+        if (lane == 0 && sum) atomicAdd(so.total, sum);
+    }
+}
+
+// ---------------------------------------------------------------- launchers
+template <typename E, int TIER, int MODE>
+static cudaError_t launch_global_m(const uint8_t *text, uint64_t n_total, const SttView &st, const Region &a,
+                                   const Region &b, const ScanOut &so, size_t smem, cudaStream_t stream) {
+    auto kern = k_scan_global<E, TIER, MODE>;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    const uint64_t threads = a.n_chains + b.n_chains;
+    const unsigned grid = (unsigned)((threads + GT - 1) / GT);
+    if (grid == 0) return cudaSuccess;
+    kern<<<grid, GT, smem, stream>>>(text, n_total, st, a, b, so);
+    return cudaGetLastError();
+}
+
+template <int TIER>
+cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint64_t n_total, const SttView &st,
+                               const Region &a, const Region &b, const ScanOut &so, size_t smem_stt,
+                               cudaStream_t stream) {
+    const size_t smem = 256 + smem_stt;
+    if (eb == 2) {
+        if (mode == MODE_COUNT_TOTAL) return launch_global_m<uint16_t, TIER, MODE_COUNT_TOTAL>(text, n_total, st, a, b, so, smem, stream);
+        if (mode == MODE_COUNT_CHAINS) return launch_global_m<uint16_t, TIER, MODE_COUNT_CHAINS>(text, n_total, st, a, b, so, smem, stream);
+        return launch_global_m<uint16_t, TIER, MODE_EMIT>(text, n_total, st, a, b, so, smem, stream);
+    }
+    if (mode == MODE_COUNT_TOTAL) return launch_global_m<uint32_t, TIER, MODE_COUNT_TOTAL>(text, n_total, st, a, b, so, smem, stream);
+    if (mode == MODE_COUNT_CHAINS) return launch_global_m<uint32_t, TIER, MODE_COUNT_CHAINS>(text, n_total, st, a, b, so, smem, stream);
+    return launch_global_m<uint32_t, TIER, MODE_EMIT>(text, n_total, st, a, b, so, smem, stream);
+}
+
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST>
+static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
+                                   const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
+    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST>;
+    const StagedConfig cfg{WARPS, K, W, NST};
+    const size_t smem = staged_smem_bytes(cfg, smem_stt);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const uint64_t R = (uint64_t)WARPS * 32 * K;
+    const unsigned grid = (unsigned)((g.n_chains + R - 1) / R);
+    if (grid == 0) return cudaSuccess;
+    kern<<<grid, WARPS * 32, smem, stream>>>(tmap, mtext, st, g, so);
+    return cudaGetLastError();
+}
+
+template <typename E, int TIER, int MODE>
+static cudaError_t launch_staged_m(int variant, const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
+                                   const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t s) {
+    switch (variant) {
+#define AC_CASE(i, w, k, wd, ns) \
+    case i: return launch_staged_v<E, TIER, MODE, w, k, wd, ns>(tmap, mtext, st, g, so, smem_stt, s);
+        AC_STAGED_VARIANTS(AC_CASE)
+#undef AC_CASE
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <int TIER>
+cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtensorMap &tmap, const uint8_t *mtext,
+                               const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
+                               cudaStream_t stream) {
+    if (eb == 2) {
+        if (mode == MODE_COUNT_TOTAL) return launch_staged_m<uint16_t, TIER, MODE_COUNT_TOTAL>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+        if (mode == MODE_COUNT_CHAINS) return launch_staged_m<uint16_t, TIER, MODE_COUNT_CHAINS>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+        return launch_staged_m<uint16_t, TIER, MODE_EMIT>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+    }
+    if (mode == MODE_COUNT_TOTAL) return launch_staged_m<uint32_t, TIER, MODE_COUNT_TOTAL>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+    if (mode == MODE_COUNT_CHAINS) return launch_staged_m<uint32_t, TIER, MODE_COUNT_CHAINS>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+    return launch_staged_m<uint32_t, TIER, MODE_EMIT>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+}
+
+}  // namespace acx

@@ -53,11 +53,20 @@ struct StagedGeom {
 };
 
 struct StagedConfig {
-    int threads;     // CTA size
-    int k;           // chains per thread
-    int width;       // tile width S in bytes (64 or 128, = TMA swizzle span)
-    int stages;      // ring depth
+    int warps;       // warps per CTA (each owns 32*k chains and a private ring)
+    int k;           // chains per lane
+    int width;       // tile width W in bytes (16 / 32 / 64 = TMA swizzle span)
+    int stages;      // ring slots per warp
 };
+
+// AC_STAGED_VARIANTS(X): X(index, warps, chains per lane, tile width, ring depth)
+#define AC_STAGED_VARIANTS(X) \
+    X(1, 16, 1, 32, 3)        \
+    X(2, 16, 2, 32, 2)        \
+    X(3, 32, 1, 32, 2)        \
+    X(4, 32, 1, 16, 3)        \
+    X(5, 16, 2, 16, 3)        \
+    X(6, 32, 2, 16, 2)
 
 // Kernel entry points (host side launchers); all return cudaError_t.
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,
@@ -71,6 +80,16 @@ cudaError_t launch_offsets(const uint64_t *counts, uint64_t n, uint64_t *chain_e
                            cudaStream_t stream);
 
 size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
+
+// per-tier instantiations (ac_tier_*.cu)
+template <int TIER>
+cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint64_t n_total, const SttView &st,
+                               const Region &a, const Region &b, const ScanOut &so, size_t smem_stt,
+                               cudaStream_t stream);
+template <int TIER>
+cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtensorMap &tmap, const uint8_t *mtext,
+                               const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
+                               cudaStream_t stream);
 int staged_variant_count();
 const StagedConfig &staged_variant(int v);  // v in [1, staged_variant_count()]
 size_t offsets_tiles(uint64_t n);
