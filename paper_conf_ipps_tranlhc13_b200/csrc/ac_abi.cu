@@ -33,8 +33,8 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
         if (e_ != cudaSuccess) return cuda_fail(e_, what); \
     } while (0)
 
-static const uint64_t kGlobalTailChain = 64;
-static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)  // head/tail chains of the staged path
+static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
+static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)
 static const uint64_t kStagedMinBytes = 64 * 1024;
 static const uint64_t kStagedMinChain = 256;
 
@@ -440,7 +440,9 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     const size_t budget = stt_budget(h, 1);  // a 48 KB-ring staged variant
     uint32_t tier = opts ? opts->tier : AC_TIER_AUTO;
     uint32_t hot = opts ? opts->hot_rows : 0;
-    if (tier == AC_TIER_AUTO) tier = stt_bytes <= budget ? AC_TIER_SMEM : AC_TIER_HYBRID;
+    // measured (scripts/sweep.py): an L1-cached global table beats a shared-memory
+    // prefix reached through generic loads, so AUTO never picks HYBRID
+    if (tier == AC_TIER_AUTO) tier = stt_bytes <= budget ? AC_TIER_SMEM : AC_TIER_GLOBAL;
     if (tier == AC_TIER_SMEM) {
         if (stt_bytes > budget) {
             delete h;

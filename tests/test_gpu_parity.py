@@ -100,7 +100,7 @@ def test_c3_hybrid_and_global_tiers():
     w = synth.make("c3", n=(1 << 20) + 5)
     o = Oracle(w.patterns)
     want = oracle_keys(o, w.text)
-    for tier in (ac.TIER_AUTO, ac.TIER_GLOBAL):
+    for tier in (ac.TIER_AUTO, ac.TIER_HYBRID, ac.TIER_GLOBAL):
         stt = ac.build(w.patterns, tier=tier)
         assert_same(gpu_keys(stt, w.text), want)
 
