@@ -75,7 +75,13 @@ typedef struct ac_stt ac_stt;
 typedef struct ac_table ac_table;
 
 /* STT residency tiers. */
-enum { AC_TIER_AUTO = 0, AC_TIER_SMEM = 1, AC_TIER_HYBRID = 2, AC_TIER_GLOBAL = 3 };
+/* SMEM: the dense table staged whole in shared memory.  HYBRID: its BFS
+ * prefix in shared memory, the rest through L1/L2.  GLOBAL: L1/L2 only.
+ * COMPACT: dense rows for shallow states + 8-byte default-transition records
+ * for the others + an output table, all in shared memory (<= 32768 states,
+ * <= 255 classes).  AUTO = SMEM if the dense table
+ * fits, else COMPACT if that fits, else GLOBAL. */
+enum { AC_TIER_AUTO = 0, AC_TIER_SMEM = 1, AC_TIER_HYBRID = 2, AC_TIER_GLOBAL = 3, AC_TIER_COMPACT = 4 };
 
 typedef struct {
     uint32_t struct_size;  /* sizeof(ac_build_opts)                          */
@@ -106,6 +112,16 @@ typedef struct {
                               else u32)                                      */
     uint64_t stt_bytes;    /* S * row_stride * entry_bytes                  */
     uint64_t out_entries;  /* sum over states of |output(s)|                */
+    /* COMPACT encoding (valid when compact_bytes != 0): byte layout
+     * [dense rows: compact_dense x compact_dstride u16]
+     * [sparse records at compact_sparse_off: (n_states - compact_dense) x 8 B,
+     *  lo32 = fd | c1 << 16 | c2 << 24, hi32 = t1 | t2 << 16]
+     * [output table at compact_out_off: (compact_od + compact_os) x
+     *  (u32 payload, u32 count)], compact ids: 0 = root, then dense output
+     * states, other dense, sparse output states, other sparse.           */
+    uint32_t compact_dense, compact_od, compact_os, compact_dstride;
+    uint32_t compact_sparse_off, compact_out_off;
+    uint64_t compact_bytes;
 } ac_stt_info;
 
 /* Scan variants (SURVEY 8(f) NEXT-1 ablations are selectable here). */
@@ -197,9 +213,12 @@ ac_status ac_match_host(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac
                         uint64_t cap, uint64_t *count, void *stream);
 
 /* ----------------------------------------------------- host-only builder
- * ac_compile: phase 1 without a device (for tests and tooling).  opts->tier
- * and hot_rows are ignored; opts->forward selects the paper's forward
- * automaton.  ac_table_export copies any non-NULL array out:
+ * ac_compile: phase 1 without a device (for tests and tooling).  hot_rows is
+ * ignored; opts->forward selects the paper's forward automaton;
+ * opts->tier == AC_TIER_COMPACT also builds the COMPACT encoding for the
+ * default shared-memory budget (AC_ERR_TOO_LARGE if it cannot).
+ * ac_table_export_compact copies it out (blob[compact_bytes], perm[S] =
+ * compact id -> dense BFS id).  ac_table_export copies any non-NULL array:
  *   class_map[256]            byte -> class
  *   stt[S * row_stride]       entries of entry_bytes each: low bits = next
  *                             state, top bit (15 or 31) = output(next) != {};
@@ -211,6 +230,7 @@ ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint3
 ac_status ac_table_query(const ac_table *t, ac_stt_info *info);
 ac_status ac_table_export(const ac_table *t, uint8_t *class_map, void *stt, uint32_t *out_off,
                           uint32_t *out_ids);
+ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm);
 void ac_table_free(ac_table *t);
 
 /* ------------------------------------------------------------ diagnostics */

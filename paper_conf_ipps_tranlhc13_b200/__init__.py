@@ -27,14 +27,14 @@ LIB_PATH = _PKG / "libac.so"
 
 AC_OK, AC_ERR_INVALID_ARG, AC_ERR_EMPTY_PATTERN, AC_ERR_TOO_LARGE = 0, 1, 2, 3
 AC_ERR_CAPACITY, AC_ERR_NO_MEMORY, AC_ERR_CUDA, AC_ERR_NO_DEVICE = 4, 5, 6, 7
-TIER_AUTO, TIER_SMEM, TIER_HYBRID, TIER_GLOBAL = 0, 1, 2, 3
+TIER_AUTO, TIER_SMEM, TIER_HYBRID, TIER_GLOBAL, TIER_COMPACT = 0, 1, 2, 3, 4
 KERNEL_AUTO, KERNEL_STAGED, KERNEL_GLOBAL = 0, 1, 2
-TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global"}
+TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global", 4: "compact"}
 
 EXPORTED = [
     "ac_build", "ac_free", "ac_stt_query", "ac_stt_pattern_lengths", "ac_match", "ac_match_shard",
     "ac_match_async", "ac_last_launch_count", "ac_last_launch_name", "ac_match_host", "ac_compile", "ac_table_query",
-    "ac_table_export", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
+    "ac_table_export", "ac_table_export_compact", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
 ]
 
 
@@ -59,7 +59,10 @@ class ac_stt_info(ctypes.Structure):
     _fields_ = [("n_patterns", ctypes.c_uint32), ("n_states", ctypes.c_uint32), ("n_classes", ctypes.c_uint32),
                 ("row_stride", ctypes.c_uint32), ("entry_bytes", ctypes.c_uint32), ("tier", ctypes.c_uint32),
                 ("hot_rows", ctypes.c_uint32), ("maxlen", ctypes.c_uint32), ("forward", ctypes.c_uint32),
-                ("info_col", ctypes.c_uint32), ("stt_bytes", ctypes.c_uint64), ("out_entries", ctypes.c_uint64)]
+                ("info_col", ctypes.c_uint32), ("stt_bytes", ctypes.c_uint64), ("out_entries", ctypes.c_uint64),
+                ("compact_dense", ctypes.c_uint32), ("compact_od", ctypes.c_uint32), ("compact_os", ctypes.c_uint32),
+                ("compact_dstride", ctypes.c_uint32), ("compact_sparse_off", ctypes.c_uint32),
+                ("compact_out_off", ctypes.c_uint32), ("compact_bytes", ctypes.c_uint64)]
 
 
 class ac_match_opts(ctypes.Structure):
@@ -89,6 +92,7 @@ def lib():
         L.ac_stt_query.argtypes = [_vp, ctypes.POINTER(ac_stt_info)]
         L.ac_table_query.argtypes = [_vp, ctypes.POINTER(ac_stt_info)]
         L.ac_table_export.argtypes = [_vp, _vp, _vp, _vp, _vp]
+        L.ac_table_export_compact.argtypes = [_vp, _vp, _vp]
         L.ac_stt_pattern_lengths.argtypes = [_vp, _vp]
         L.ac_match.argtypes = [_vp, _vp, _u64, _vp, _u64, _u64p, _vp]
         L.ac_match_shard.argtypes = [_vp, _vp, _u64, _u64, _u64, _vp, _u64, _u64p, _vp]
@@ -305,15 +309,17 @@ class HostTable:
     stt: "object"
     out_off: "object"
     out_ids: "object"
+    compact: "object" = None   # COMPACT blob (uint8) if requested
+    perm: "object" = None      # compact id -> dense BFS id
 
 
-def compile_table(patterns, forward: bool = False, entry_bytes: int = 0) -> HostTable:
+def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact: bool = False) -> HostTable:
     """Phase 1 on the host only (no device) -- for builder tests."""
     import numpy as np
     L = lib()
     pats, bufs, ptrs, lens = _pattern_arrays(patterns)
     h = ctypes.c_void_p()
-    o = _opts(entry_bytes=entry_bytes, forward=forward)
+    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=TIER_COMPACT if compact else TIER_AUTO)
     _check(L.ac_compile(ptrs, lens, len(pats), ctypes.byref(o), ctypes.byref(h)))
     try:
         info = ac_stt_info()
@@ -325,6 +331,11 @@ def compile_table(patterns, forward: bool = False, entry_bytes: int = 0) -> Host
         off = np.zeros(d["n_states"] + 1, dtype=np.uint32)
         ids = np.zeros(max(1, d["out_entries"]), dtype=np.uint32)
         _check(L.ac_table_export(h, cm.ctypes.data, stt.ctypes.data, off.ctypes.data, ids.ctypes.data))
-        return HostTable(d, cm, stt.reshape(d["n_states"], d["row_stride"]), off, ids[:d["out_entries"]])
+        blob = perm = None
+        if compact:
+            blob = np.zeros(d["compact_bytes"], dtype=np.uint8)
+            perm = np.zeros(d["n_states"], dtype=np.uint32)
+            _check(L.ac_table_export_compact(h, blob.ctypes.data, perm.ctypes.data))
+        return HostTable(d, cm, stt.reshape(d["n_states"], d["row_stride"]), off, ids[:d["out_entries"]], blob, perm)
     finally:
         L.ac_table_free(h)

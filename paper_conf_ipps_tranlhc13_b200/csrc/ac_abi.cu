@@ -35,6 +35,10 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
 
 static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
 static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)
+static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slots (32 KB ring)
+// COMPACT budget used by ac_compile (no device): B200's 227 KB opt-in shared
+// memory minus the lean staged variant's ring and bookkeeping (= stt_budget)
+#define kDefaultCompactBudget (232448 - staged_smem_bytes(staged_variant(kLeanVariant), 0) - 1024)
 static const uint64_t kStagedMinBytes = 64 * 1024;
 static const uint64_t kStagedMinChain = 256;
 
@@ -106,18 +110,28 @@ static SttView view_of(const ac_stt *h, int v) {
     s.n_states = h->host.n_states;
     s.halo = h->host.maxlen ? h->host.maxlen - 1 : 0;
     s.info_col = h->host.info_col;
+    s.c_dense = h->host.c_dense;
+    s.c_od = h->host.c_od;
+    s.c_dstride = h->host.c_dstride;
+    s.c_sparse_off = h->host.c_sparse_off;
+    s.c_out_off = h->host.c_out_off;
+    if (h->tier == AC_TIER_COMPACT) {
+        s.smem_rows = h->host.n_states;
+        s.smem_bytes = (uint32_t)h->host.compact.size();
+        return s;
+    }
     uint64_t rows = h->tier == AC_TIER_GLOBAL ? 0 : h->hot_rows;
     const uint64_t cap = stt_budget(h, v) / row_bytes(h);
     s.smem_rows = (uint32_t)(rows < cap ? rows : cap);
+    s.smem_bytes = (uint32_t)(s.smem_rows * row_bytes(h));
     return s;
 }
 
-static size_t smem_of(const ac_stt *h, const SttView &v) {
-    return ((size_t)v.smem_rows * row_bytes(h) + 15) / 16 * 16;
-}
+static size_t smem_of(const ac_stt *, const SttView &v) { return ((size_t)v.smem_bytes + 15) / 16 * 16; }
 
 // The kernel's tier: SMEM only when every row is resident, GLOBAL when none.
 static uint32_t tier_of(const ac_stt *h, const SttView &v) {
+    if (h->tier == AC_TIER_COMPACT) return AC_TIER_COMPACT;
     if (v.smem_rows == 0) return AC_TIER_GLOBAL;
     if (v.smem_rows >= h->host.n_states) return AC_TIER_SMEM;
     return AC_TIER_HYBRID;
@@ -179,7 +193,14 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         set_error("unknown staged variant");
         return AC_ERR_INVALID_ARG;
     }
-    if (variant == 0) variant = kAutoVariant;
+    if (variant == 0) {
+        variant = kAutoVariant;
+        if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
+    }
+    if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, variant)) {
+        set_error("staged variant " + std::to_string(variant) + " has no room for the COMPACT table");
+        return AC_ERR_INVALID_ARG;
+    }
     const SttView sg = view_of(h, 0), ss = view_of(h, variant);
     const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
     const size_t smem_g = smem_of(h, sg), smem_s = smem_of(h, ss);
@@ -349,6 +370,10 @@ ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint3
     ac_status rc;
     try {
         rc = compile_table(patterns, lens, n, opts, *t);
+        if (rc == AC_OK && opts && opts->tier == AC_TIER_COMPACT && !compact_table(*t, kDefaultCompactBudget)) {
+            set_error("the automaton does not fit the COMPACT shared-memory encoding");
+            rc = AC_ERR_TOO_LARGE;
+        }
     } catch (...) {
         set_error("host allocation failed");
         rc = AC_ERR_NO_MEMORY;
@@ -373,6 +398,20 @@ static void fill_info(const ac_table &t, ac_stt_info *info) {
     info->info_col = t.info_col;
     info->stt_bytes = (uint64_t)t.n_states * t.row_stride * t.entry_bytes;
     info->out_entries = t.out_ids.size();
+    info->compact_dense = t.c_dense;
+    info->compact_od = t.c_od;
+    info->compact_os = t.c_os;
+    info->compact_dstride = t.c_dstride;
+    info->compact_sparse_off = t.c_sparse_off;
+    info->compact_out_off = t.c_out_off;
+    info->compact_bytes = t.compact.size();
+}
+
+ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm) {
+    if (!t || t->compact.empty()) return AC_ERR_INVALID_ARG;
+    if (blob) std::memcpy(blob, t->compact.data(), t->compact.size());
+    if (perm) std::memcpy(perm, t->c_perm.data(), t->c_perm.size() * 4);
+    return AC_OK;
 }
 
 ac_status ac_table_query(const ac_table *t, ac_stt_info *info) {
@@ -407,7 +446,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
         set_error("the device scan needs the reversed automaton (forward=0)");
         return AC_ERR_INVALID_ARG;
     }
-    if (opts && opts->tier > AC_TIER_GLOBAL) {
+    if (opts && opts->tier > AC_TIER_COMPACT) {
         set_error("unknown tier");
         return AC_ERR_INVALID_ARG;
     }
@@ -442,8 +481,20 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     uint32_t hot = opts ? opts->hot_rows : 0;
     // measured (scripts/sweep.py): an L1-cached global table beats a shared-memory
     // prefix reached through generic loads, so AUTO never picks HYBRID
-    if (tier == AC_TIER_AUTO) tier = stt_bytes <= budget ? AC_TIER_SMEM : AC_TIER_GLOBAL;
-    if (tier == AC_TIER_SMEM) {
+    const size_t cbudget = stt_budget(h, kLeanVariant);
+    if (tier == AC_TIER_AUTO) {
+        if (stt_bytes <= budget) tier = AC_TIER_SMEM;
+        else if (compact_table(h->host, cbudget)) tier = AC_TIER_COMPACT;
+        else tier = AC_TIER_GLOBAL;
+    }
+    if (tier == AC_TIER_COMPACT) {
+        if (h->host.compact.empty() && !compact_table(h->host, cbudget)) {
+            delete h;
+            set_error("the automaton does not fit the COMPACT shared-memory encoding");
+            return AC_ERR_TOO_LARGE;
+        }
+        hot = t.n_states;
+    } else if (tier == AC_TIER_SMEM) {
         if (stt_bytes > budget) {
             delete h;
             set_error("STT (" + std::to_string(stt_bytes) + " B) does not fit shared memory (" +
@@ -472,10 +523,11 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     };
     cudaError_t e = cudaSetDevice(device);
     if (e != cudaSuccess) return fail(e, "cudaSetDevice");
-    const size_t stt_alloc = (stt_bytes + 15) / 16 * 16 + 16;
+    const std::vector<uint8_t> &blob = tier == AC_TIER_COMPACT ? t.compact : t.stt;
+    const size_t stt_alloc = (blob.size() + 15) / 16 * 16 + 16;
     if ((e = cudaMalloc(&h->d_stt, stt_alloc)) != cudaSuccess) return fail(e, "cudaMalloc(stt)");
     if ((e = cudaMemset(h->d_stt, 0, stt_alloc)) != cudaSuccess) return fail(e, "cudaMemset(stt)");
-    if ((e = cudaMemcpy(h->d_stt, t.stt.data(), stt_bytes, cudaMemcpyHostToDevice)) != cudaSuccess)
+    if ((e = cudaMemcpy(h->d_stt, blob.data(), blob.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
         return fail(e, "H2D stt");
     if ((e = cudaMalloc(&h->d_class_map, 256)) != cudaSuccess) return fail(e, "cudaMalloc(class map)");
     if ((e = cudaMemcpy(h->d_class_map, t.class_map, 256, cudaMemcpyHostToDevice)) != cudaSuccess)

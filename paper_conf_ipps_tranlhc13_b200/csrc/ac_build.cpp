@@ -112,8 +112,7 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
         // ---- BFS order, failure function and delta (AC'75 Alg. 3/4)
         std::vector<uint32_t> order;
         order.reserve(S);
-        std::vector<uint32_t> fail(S, 0);
-        std::vector<uint8_t> is_child(C);
+        std::vector<uint32_t> fail(S, 0), depth(S, 0);
         order.push_back(0);
         for (size_t qi = 0; qi < order.size(); qi++) {
             uint32_t r = order[qi];
@@ -122,6 +121,7 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
                 int32_t child = row[c];
                 if (child >= 0) {
                     order.push_back((uint32_t)child);
+                    depth[child] = depth[r] + 1;
                     fail[child] = (r == 0) ? 0u : (uint32_t)(go[(size_t)fail[r] * C + c] & 0x7fffffff);
                     row[c] = child;
                 } else {
@@ -147,6 +147,12 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
         // ---- renumber in BFS order
         std::vector<uint32_t> rank(S);
         for (uint32_t i = 0; i < S; i++) rank[order[i]] = i;
+        t.fail.resize(S);
+        t.depth.resize(S);
+        for (uint32_t i = 0; i < S; i++) {
+            t.fail[i] = rank[fail[order[i]]];
+            t.depth[i] = depth[order[i]];
+        }
         uint32_t eb = want_eb ? want_eb : (S <= 32768 ? 2u : 4u);
         if (eb == 2 && S > 32768) {
             set_error("entry_bytes=2 needs <= 32768 states");

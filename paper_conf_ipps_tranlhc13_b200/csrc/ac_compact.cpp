@@ -1,0 +1,160 @@
+// ac_compact.cpp -- the COMPACT STT encoding.
+//
+// The paper keeps the whole STT in texture memory and notes that its cache
+// misses grow with the number of patterns.  On sm_100a the
+// fast tier is shared memory, but a dense AC table for ~1,000 English
+// patterns (15K states x 31 classes x 2 B) is ~1 MB.  Most of those rows are
+// near-copies: in the AC automaton delta(s,c) = g(s,c) if the trie has that
+// edge, else delta(f(s),c) (P:62 with the failure function of P:52), and a
+// deep trie state almost always has a single child.  So:
+//
+//   * DENSE states (the BFS prefix up to depth d, plus any state that needs
+//     more than two exceptions) keep a full row of C entries.
+//   * Every other (SPARSE) state s gets an 8-byte record: fd(s) = the first
+//     dense state on its failure chain, and up to two exceptions (c, delta(s,c))
+//     -- exactly the classes where delta(s,.) differs from delta(fd(s),.).
+//     delta(s,c) = exception if c matches one, else dense[fd(s)][c]: at most
+//     two shared-memory loads per byte, no loop.
+//   * Output states are numbered first inside each group so the output
+//     table index is arithmetic: oidx = x - 1 (dense, x >= 1) or
+//     c_od + x - c_dense (sparse); each table slot holds (payload, count)
+//     exactly like the dense rows' output summary.
+//
+// Entries keep the dense layout's convention: bit 15 = output(next) != {},
+// bits 0..14 = next state (COMPACT requires <= 32768 states and C <= 255).
+#include <algorithm>
+#include <cstring>
+
+#include "ac_internal.h"
+
+namespace acx {
+
+size_t compact_bytes_for(const ac_table &t, uint32_t d, std::vector<uint8_t> *dense_out, uint32_t *n_dense) {
+    const uint32_t S = t.n_states, C = t.n_classes, stride = t.row_stride;
+    auto delta = [&](uint32_t s, uint32_t c) -> uint32_t {
+        uint16_t e;
+        std::memcpy(&e, &t.stt[((size_t)s * stride + c) * 2], 2);
+        return e & 0x7fffu;
+    };
+    std::vector<uint8_t> dense(S, 0);
+    std::vector<uint32_t> fd(S, 0);
+    uint32_t nd = 0;
+    for (uint32_t s = 0; s < S; s++) {  // BFS order: f(s) is decided before s
+        if (s == 0 || t.depth[s] <= d) {
+            dense[s] = 1;
+        } else {
+            const uint32_t f = t.fail[s];
+            fd[s] = dense[f] ? f : fd[f];
+            uint32_t exc = 0;
+            for (uint32_t c = 0; c < C && exc <= 2; c++) exc += delta(s, c) != delta(fd[s], c);
+            if (exc > 2) dense[s] = 1;
+        }
+        nd += dense[s];
+    }
+    uint32_t words = (C + 1) / 2;
+    if (words % 2 == 0) words++;
+    uint32_t n_out = 0;
+    for (uint32_t s = 0; s < S; s++) n_out += t.out_off[s + 1] > t.out_off[s];
+    if (dense_out) dense_out->swap(dense);
+    if (n_dense) *n_dense = nd;
+    const size_t dense_bytes = (size_t)nd * words * 4;
+    return (dense_bytes + 7) / 8 * 8 + (size_t)(S - nd) * 8 + (size_t)n_out * 8;
+}
+
+// Build the COMPACT encoding into t.compact if it fits `budget` bytes.
+// Returns false (t unchanged) when the automaton cannot be compacted.
+bool compact_table(ac_table &t, size_t budget) {
+    const uint32_t S = t.n_states, C = t.n_classes, stride = t.row_stride;
+    if (t.entry_bytes != 2 || S > 32768 || C > 255 || S == 0) return false;
+    uint32_t maxd = 0;
+    for (uint32_t s = 0; s < S; s++) maxd = std::max(maxd, t.depth[s]);
+    // the deepest dense prefix that fits (the size is not monotonic in d:
+    // shallow prefixes force many states with > 2 exceptions to be dense)
+    int best = -1;
+    for (uint32_t d = 0; d <= maxd; d++)
+        if (compact_bytes_for(t, d, nullptr, nullptr) <= budget) best = (int)d;
+    if (best < 0) return false;
+    std::vector<uint8_t> dense;
+    uint32_t nd = 0;
+    const size_t total = compact_bytes_for(t, (uint32_t)best, &dense, &nd);
+    auto delta_e = [&](uint32_t s, uint32_t c) -> uint16_t {
+        uint16_t e;
+        std::memcpy(&e, &t.stt[((size_t)s * stride + c) * 2], 2);
+        return e;
+    };
+    auto is_out = [&](uint32_t s) { return t.out_off[s + 1] > t.out_off[s]; };
+    // numbering: root, dense outputs, other dense, sparse outputs, other sparse
+    std::vector<uint32_t> perm;  // compact id -> BFS id
+    perm.reserve(S);
+    perm.push_back(0);
+    uint32_t od = 0, os = 0;
+    for (uint32_t s = 1; s < S; s++)
+        if (dense[s] && is_out(s)) perm.push_back(s), od++;
+    for (uint32_t s = 1; s < S; s++)
+        if (dense[s] && !is_out(s)) perm.push_back(s);
+    for (uint32_t s = 1; s < S; s++)
+        if (!dense[s] && is_out(s)) perm.push_back(s), os++;
+    for (uint32_t s = 1; s < S; s++)
+        if (!dense[s] && !is_out(s)) perm.push_back(s);
+    std::vector<uint32_t> inv(S);
+    for (uint32_t x = 0; x < S; x++) inv[perm[x]] = x;
+    auto enc = [&](uint16_t e) -> uint16_t { return (uint16_t)(inv[e & 0x7fffu] | (e & 0x8000u)); };
+
+    uint32_t words = (C + 1) / 2;
+    if (words % 2 == 0) words++;
+    const uint32_t dstride = words * 2;
+    const size_t dense_bytes = ((size_t)nd * dstride * 2 + 7) / 8 * 8;
+    std::vector<uint8_t> blob(total, 0);
+    for (uint32_t x = 0; x < nd; x++) {
+        const uint32_t s = perm[x];
+        for (uint32_t c = 0; c < C; c++) {
+            const uint16_t e = enc(delta_e(s, c));
+            std::memcpy(&blob[((size_t)x * dstride + c) * 2], &e, 2);
+        }
+    }
+    // sparse records: lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
+    std::vector<uint32_t> fd(S, 0);
+    for (uint32_t s = 1; s < S; s++)
+        if (!dense[s]) fd[s] = dense[t.fail[s]] ? t.fail[s] : fd[t.fail[s]];
+    for (uint32_t x = nd; x < S; x++) {
+        const uint32_t s = perm[x];
+        uint32_t cls[2] = {0xFF, 0xFF};
+        uint16_t tgt[2] = {0, 0};
+        uint32_t k = 0;
+        for (uint32_t c = 0; c < C; c++) {
+            const uint16_t e = delta_e(s, c);
+            if ((e & 0x7fffu) != (delta_e(fd[s], c) & 0x7fffu)) {
+                cls[k] = c;
+                tgt[k] = enc(e);
+                k++;
+            }
+        }
+        const uint32_t lo = inv[fd[s]] | (cls[0] << 16) | (cls[1] << 24);
+        const uint32_t hi = (uint32_t)tgt[0] | ((uint32_t)tgt[1] << 16);
+        uint8_t *r = &blob[dense_bytes + (size_t)(x - nd) * 8];
+        std::memcpy(r, &lo, 4);
+        std::memcpy(r + 4, &hi, 4);
+    }
+    // output table
+    const size_t out_base = dense_bytes + (size_t)(S - nd) * 8;
+    auto put_out = [&](uint32_t oidx, uint32_t s) {
+        const uint32_t a = t.out_off[s], z = t.out_off[s + 1];
+        const uint32_t payload = (z - a == 1) ? t.out_ids[a] : a, count = z - a;
+        std::memcpy(&blob[out_base + (size_t)oidx * 8], &payload, 4);
+        std::memcpy(&blob[out_base + (size_t)oidx * 8 + 4], &count, 4);
+    };
+    for (uint32_t i = 0; i < od; i++) put_out(i, perm[1 + i]);
+    for (uint32_t i = 0; i < os; i++) put_out(od + i, perm[nd + i]);
+
+    t.compact.swap(blob);
+    t.c_perm.swap(perm);
+    t.c_dense = nd;
+    t.c_od = od;
+    t.c_os = os;
+    t.c_dstride = dstride;
+    t.c_sparse_off = (uint32_t)dense_bytes;
+    t.c_out_off = (uint32_t)out_base;
+    return true;
+}
+
+}  // namespace acx

@@ -22,6 +22,18 @@ struct ac_table {
     std::vector<uint32_t> out_off;     // n_states + 1
     std::vector<uint32_t> out_ids;     // output CSR (ids ascending per state)
     std::vector<uint32_t> lens;        // pattern lengths
+    std::vector<uint32_t> fail;        // failure function, BFS ids
+    std::vector<uint32_t> depth;       // state depth (trie level)
+
+    // COMPACT encoding, built by compact_table():
+    //   [dense rows: c_dense x c_dstride u16][sparse records: (S - c_dense) x 8 B][output table: n_out x 8 B]
+    // in its own numbering: 0 = root, [1, 1 + c_od) = dense output states,
+    // then the other dense states, [c_dense, c_dense + c_os) = sparse output
+    // states, then the other sparse states.
+    uint32_t c_dense = 0, c_od = 0, c_os = 0, c_dstride = 0;
+    uint32_t c_sparse_off = 0, c_out_off = 0;  // byte offsets inside `compact`
+    std::vector<uint8_t> compact;
+    std::vector<uint32_t> c_perm;              // compact id -> BFS id
 };
 
 // Device-side STT (library owned).
@@ -43,4 +55,5 @@ namespace acx {
 void set_error(const std::string &msg);
 ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n,
                         const ac_build_opts *opts, ac_table &t);
+bool compact_table(ac_table &t, size_t budget);
 }  // namespace acx

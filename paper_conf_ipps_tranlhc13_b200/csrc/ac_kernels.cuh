@@ -64,7 +64,7 @@ __device__ __forceinline__ void stage_tables(uint8_t *s_cmap, E *s_stt, const St
     const uint4 *c4 = reinterpret_cast<const uint4 *>(st.cmap);
     uint4 *d4 = reinterpret_cast<uint4 *>(s_cmap);
     for (int i = threadIdx.x; i < 16; i += blockDim.x) d4[i] = __ldg(c4 + i);
-    const size_t words = ((size_t)st.smem_rows * st.stride * sizeof(E) + 15) / 16;
+    const size_t words = ((size_t)st.smem_bytes + 15) / 16;
     const uint4 *src = reinterpret_cast<const uint4 *>(st.stt);
     uint4 *dst = reinterpret_cast<uint4 *>(s_stt);
     for (size_t i = threadIdx.x; i < words; i += blockDim.x) dst[i] = __ldg(src + i);
@@ -83,14 +83,36 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
     }
 }
 
+// The entry delta(s, cls): next state in the low bits, output flag on top.
+// COMPACT: a dense row, or a sparse record's exception, or the dense row of
+// the record's default state fd(s) -- at most two shared-memory loads.
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t next_entry(const E *s_stt, const SttView &st, uint32_t s, uint32_t cls) {
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        const uint16_t *dense = reinterpret_cast<const uint16_t *>(s_stt);
+        if (s < st.c_dense) return dense[s * st.c_dstride + cls];
+        const uint2 r = reinterpret_cast<const uint2 *>(reinterpret_cast<const uint8_t *>(s_stt) +
+                                                        st.c_sparse_off)[s - st.c_dense];
+        if (cls == ((r.x >> 16) & 0xFFu)) return r.y & 0xFFFFu;
+        if (cls == (r.x >> 24)) return r.y >> 16;
+        return dense[(r.x & 0xFFFFu) * st.c_dstride + cls];
+    } else {
+        return stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
+    }
+}
+
 // One transition with no output (halo warm-up).
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uint8_t *s_cmap, const E *s_stt,
                                             const SttView &st) {
-    const uint32_t cls = s_cmap[byte];
-    const uint32_t e =
-        stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
-    return e & EntryBits<E>::MASK;
+    return next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]) & EntryBits<E>::MASK;
+}
+
+// COMPACT output table slot of output state s: (payload, count).
+template <typename E>
+__device__ __forceinline__ uint2 compact_out(const E *s_stt, const SttView &st, uint32_t s) {
+    const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
+    return reinterpret_cast<const uint2 *>(reinterpret_cast<const uint8_t *>(s_stt) + st.c_out_off)[oidx];
 }
 
 // Output summary of state s, stored in the padding of its own STT row
@@ -99,23 +121,31 @@ __device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uin
 // common single-output case.
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t out_count(const E *s_stt, const SttView &st, uint32_t s) {
-    const uint32_t idx = s * st.stride + st.info_col + (sizeof(E) == 2 ? 2 : 1);
-    uint32_t c = stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, idx);
-    if (sizeof(E) == 2 && c == 0xFFFFu) c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);
-    return c;
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return compact_out<E>(s_stt, st, s).y;
+    } else {
+        const uint32_t idx = s * st.stride + st.info_col + (sizeof(E) == 2 ? 2 : 1);
+        uint32_t c = stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, idx);
+        if (sizeof(E) == 2 && c == 0xFFFFu) c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);
+        return c;
+    }
 }
 
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t out_payload(const E *s_stt, const SttView &st, uint32_t s) {
-    const uint32_t idx = s * st.stride + st.info_col;  // 4-byte aligned by construction
-    const uint32_t *sp = reinterpret_cast<const uint32_t *>(s_stt + idx);
-    const uint32_t *gp = reinterpret_cast<const uint32_t *>(static_cast<const E *>(st.stt) + idx);
-    if constexpr (TIER == AC_TIER_SMEM) {
-        return *sp;
-    } else if constexpr (TIER == AC_TIER_GLOBAL) {
-        return __ldg(gp);
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return compact_out<E>(s_stt, st, s).x;
     } else {
-        return *((s < st.smem_rows) ? sp : gp);
+        const uint32_t idx = s * st.stride + st.info_col;  // 4-byte aligned by construction
+        const uint32_t *sp = reinterpret_cast<const uint32_t *>(s_stt + idx);
+        const uint32_t *gp = reinterpret_cast<const uint32_t *>(static_cast<const E *>(st.stt) + idx);
+        if constexpr (TIER == AC_TIER_SMEM) {
+            return *sp;
+        } else if constexpr (TIER == AC_TIER_GLOBAL) {
+            return __ldg(gp);
+        } else {
+            return *((s < st.smem_rows) ? sp : gp);
+        }
     }
 }
 
@@ -124,9 +154,7 @@ template <typename E, int TIER, int MODE>
 __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp, uint32_t byte, uint64_t pos,
                                         bool live, const uint8_t *s_cmap, const E *s_stt, const SttView &st,
                                         const ScanOut &so) {
-    const uint32_t cls = s_cmap[byte];
-    const uint32_t e =
-        stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
+    const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
     s = e & EntryBits<E>::MASK;
     if ((e & EntryBits<E>::FLAG) && live) {
         const uint32_t c = out_count<E, TIER>(s_stt, st, s);
@@ -422,6 +450,7 @@ cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint6
         if (mode == MODE_COUNT_CHAINS) return launch_global_m<uint16_t, TIER, MODE_COUNT_CHAINS>(text, n_total, st, a, b, so, smem, stream);
         return launch_global_m<uint16_t, TIER, MODE_EMIT>(text, n_total, st, a, b, so, smem, stream);
     }
+    if constexpr (TIER == AC_TIER_COMPACT) return cudaErrorInvalidValue;  // COMPACT is 16-bit only
     if (mode == MODE_COUNT_TOTAL) return launch_global_m<uint32_t, TIER, MODE_COUNT_TOTAL>(text, n_total, st, a, b, so, smem, stream);
     if (mode == MODE_COUNT_CHAINS) return launch_global_m<uint32_t, TIER, MODE_COUNT_CHAINS>(text, n_total, st, a, b, so, smem, stream);
     return launch_global_m<uint32_t, TIER, MODE_EMIT>(text, n_total, st, a, b, so, smem, stream);
@@ -463,6 +492,7 @@ cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtenso
         if (mode == MODE_COUNT_CHAINS) return launch_staged_m<uint16_t, TIER, MODE_COUNT_CHAINS>(variant, tmap, mtext, st, g, so, smem_stt, stream);
         return launch_staged_m<uint16_t, TIER, MODE_EMIT>(variant, tmap, mtext, st, g, so, smem_stt, stream);
     }
+    if constexpr (TIER == AC_TIER_COMPACT) return cudaErrorInvalidValue;  // COMPACT is 16-bit only
     if (mode == MODE_COUNT_TOTAL) return launch_staged_m<uint32_t, TIER, MODE_COUNT_TOTAL>(variant, tmap, mtext, st, g, so, smem_stt, stream);
     if (mode == MODE_COUNT_CHAINS) return launch_staged_m<uint32_t, TIER, MODE_COUNT_CHAINS>(variant, tmap, mtext, st, g, so, smem_stt, stream);
     return launch_staged_m<uint32_t, TIER, MODE_EMIT>(variant, tmap, mtext, st, g, so, smem_stt, stream);

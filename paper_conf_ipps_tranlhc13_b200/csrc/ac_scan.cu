@@ -29,6 +29,7 @@ cudaError_t launch_scan_global(int mode, uint32_t eb, uint32_t tier, const uint8
     switch (tier) {
         case AC_TIER_SMEM: return launch_global_tier<AC_TIER_SMEM>(mode, eb, text, n_total, st, a, b, so, smem_stt, stream);
         case AC_TIER_HYBRID: return launch_global_tier<AC_TIER_HYBRID>(mode, eb, text, n_total, st, a, b, so, smem_stt, stream);
+        case AC_TIER_COMPACT: return launch_global_tier<AC_TIER_COMPACT>(mode, eb, text, n_total, st, a, b, so, smem_stt, stream);
         default: return launch_global_tier<AC_TIER_GLOBAL>(mode, eb, text, n_total, st, a, b, so, smem_stt, stream);
     }
 }
@@ -39,6 +40,7 @@ cudaError_t launch_scan_staged(int mode, uint32_t eb, uint32_t tier, int variant
     switch (tier) {
         case AC_TIER_SMEM: return launch_staged_tier<AC_TIER_SMEM>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
         case AC_TIER_HYBRID: return launch_staged_tier<AC_TIER_HYBRID>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
+        case AC_TIER_COMPACT: return launch_staged_tier<AC_TIER_COMPACT>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
         default: return launch_staged_tier<AC_TIER_GLOBAL>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
     }
 }

@@ -23,6 +23,9 @@ struct SttView {
     uint32_t smem_rows;       // rows staged into shared memory
     uint32_t halo;            // maxlen - 1
     uint32_t info_col;        // entry index of the row's output summary (payload u32, count)
+    uint32_t smem_bytes;      // STT bytes staged into shared memory
+    // COMPACT tier (ac_compact.cpp): dense/sparse split and blob offsets
+    uint32_t c_dense, c_od, c_dstride, c_sparse_off, c_out_off;
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.
@@ -66,7 +69,8 @@ struct StagedConfig {
     X(3, 32, 1, 32, 2)        \
     X(4, 32, 1, 16, 3)        \
     X(5, 16, 2, 16, 3)        \
-    X(6, 32, 2, 16, 2)
+    X(6, 32, 2, 16, 2)        \
+    X(7, 32, 1, 16, 2)
 
 // Kernel entry points (host side launchers); all return cudaError_t.
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,

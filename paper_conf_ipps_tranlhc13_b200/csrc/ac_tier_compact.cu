@@ -1,0 +1,11 @@
+// ac_tier_compact.cu -- instantiates the scan kernels for the COMPACT STT tier.
+#include "ac_kernels.cuh"
+
+namespace acx {
+template cudaError_t launch_global_tier<AC_TIER_COMPACT>(int, uint32_t, const uint8_t *, uint64_t, const SttView &,
+                                                     const Region &, const Region &, const ScanOut &, size_t,
+                                                     cudaStream_t);
+template cudaError_t launch_staged_tier<AC_TIER_COMPACT>(int, uint32_t, int, const CUtensorMap &, const uint8_t *,
+                                                     const SttView &, const StagedGeom &, const ScanOut &, size_t,
+                                                     cudaStream_t);
+}  // namespace acx

@@ -35,7 +35,7 @@ def main():
     p = argparse.ArgumentParser()
     p.add_argument("--config", default="c2")
     p.add_argument("--n", type=int, default=0)
-    p.add_argument("--variants", default="1,2,3,4,5")
+    p.add_argument("--variants", default="1,2,3,4,5,6,7")
     p.add_argument("--tiers", default="auto")
     p.add_argument("--global-kernel", action="store_true")
     a = p.parse_args()
@@ -43,7 +43,8 @@ def main():
     n = w.text.size
     text = torch.from_numpy(w.text).cuda()
     res = torch.zeros(2, dtype=torch.int64, device="cuda")
-    tiers = {"auto": ac.TIER_AUTO, "smem": ac.TIER_SMEM, "hybrid": ac.TIER_HYBRID, "global": ac.TIER_GLOBAL}
+    tiers = {"auto": ac.TIER_AUTO, "smem": ac.TIER_SMEM, "hybrid": ac.TIER_HYBRID, "global": ac.TIER_GLOBAL,
+             "compact": ac.TIER_COMPACT}
     for tname in a.tiers.split(","):
         stt = ac.build(w.patterns, tier=tiers[tname])
         cnt = ac.count(stt, text)
@@ -54,6 +55,11 @@ def main():
         ref = None
         for kernel, v in settings:
             knobs = dict(kernel=kernel, variant=v)
+            try:
+                ac.match_async(stt, text, None, res, **knobs)
+            except ac.AcError as e:
+                print(json.dumps({"config": a.config, "variant": v, "skipped": str(e)}), flush=True)
+                continue
             t_count = timeit(lambda: ac.match_async(stt, text, None, res, **knobs))
             t_list = timeit(lambda: ac.match_async(stt, text, out, res, **knobs))
             torch.cuda.synchronize()

@@ -96,6 +96,36 @@ def test_tiers_and_widths(tier, hot, eb):
         assert_same(gpu_keys(stt, w.text, kernel=k), want)
 
 
+@pytest.mark.parametrize("variant", [0, 4, 7])
+@pytest.mark.parametrize("name,n,P", [("c2", 3 << 20, None), ("c1", 1 << 20, None), ("c2", 1 << 20, 60)])
+def test_compact_tier(name, n, P, variant):
+    w = synth.make(name, n=n + 999, n_patterns=P)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns, tier=ac.TIER_COMPACT)
+    assert stt.tier_name == "compact"
+    want = oracle_keys(o, w.text)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
+    if variant == 0:
+        assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_GLOBAL), want)
+
+
+def test_compact_is_auto_for_c2():
+    w = synth.make("c2", n=1 << 20)
+    stt = ac.build(w.patterns)
+    assert stt.tier_name == "compact" and stt.info["n_states"] > 15000
+
+
+def test_compact_edge_cases():
+    pats = [b"he", b"she", b"his", b"hers", b"\x00\x00", b"a" * 40, b"ab" * 10]
+    o = Oracle(pats)
+    stt = ac.build(pats, tier=ac.TIER_COMPACT)
+    rng = np.random.default_rng(9)
+    text = rng.choice(np.frombuffer(b"hersia\x00b", np.uint8), size=(1 << 20) + 3)
+    text[5000:5040] = ord("a")
+    for k in KERNELS:
+        assert_same(gpu_keys(stt, text, kernel=k), oracle_keys(o, text))
+
+
 def test_c3_hybrid_and_global_tiers():
     w = synth.make("c3", n=(1 << 20) + 5)
     o = Oracle(w.patterns)

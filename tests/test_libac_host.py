@@ -144,6 +144,61 @@ def test_builder_snort_like_entry4():
     _check_builder(pats, False)
 
 
+def _decode_compact(t):
+    """The COMPACT lookup rule of include/ac.h, vectorised: returns the entry
+    table E[x, c] (compact ids, bit 15 = output flag) and the output table."""
+    d = t.info
+    S, C = d["n_states"], d["n_classes"]
+    nd, ds = d["compact_dense"], d["compact_dstride"]
+    blob = t.compact
+    dense = blob[:nd * ds * 2].view(np.uint16).reshape(nd, ds)[:, :C].astype(np.int64)
+    rec = blob[d["compact_sparse_off"]:d["compact_sparse_off"] + (S - nd) * 8].view(np.uint32).reshape(-1, 2)
+    fd = rec[:, 0] & 0xFFFF
+    c1, c2 = (rec[:, 0] >> 16) & 0xFF, rec[:, 0] >> 24
+    t1, t2 = rec[:, 1] & 0xFFFF, rec[:, 1] >> 16
+    cls = np.arange(C)[None, :]
+    sparse = np.where(cls == c1[:, None], t1[:, None],
+                      np.where(cls == c2[:, None], t2[:, None], dense[fd]))
+    E = np.concatenate([dense, sparse.astype(np.int64)])
+    nout = d["compact_od"] + d["compact_os"]
+    ot = blob[d["compact_out_off"]:d["compact_out_off"] + nout * 8].view(np.uint32).reshape(-1, 2)
+    return E, ot
+
+
+@pytest.mark.parametrize("which", ["c2", "c1", "tiny"])
+def test_compact_encoding_equals_dense(which):
+    import synth
+    if which == "tiny":
+        pats = [b"he", b"she", b"his", b"hers", b"h", b"hershey"]
+    else:
+        pats = synth.make(which, n=1 << 16).patterns if which == "c1" else synth.make("c2", n=1 << 22).patterns
+    t = ac.compile_table(pats, compact=True)
+    d = t.info
+    S, C = d["n_states"], d["n_classes"]
+    perm = t.perm.astype(np.int64)
+    assert perm[0] == 0 and sorted(perm.tolist()) == list(range(S))
+    inv = np.empty(S, np.int64)
+    inv[perm] = np.arange(S)
+    E, ot = _decode_compact(t)
+    dense_bfs = t.stt[:, :C].astype(np.int64)
+    want = inv[dense_bfs[perm] & 0x7FFF] | (dense_bfs[perm] & 0x8000)
+    assert np.array_equal(E, want)
+    # output-state numbering and the output table
+    nd, od, os_ = d["compact_dense"], d["compact_od"], d["compact_os"]
+    has_out = np.diff(t.out_off.astype(np.int64))[perm] > 0
+    assert has_out[1:1 + od].all() and not has_out[1 + od:nd].any()
+    assert has_out[nd:nd + os_].all() and not has_out[nd + os_:].any() and not has_out[0]
+    for x in list(range(1, 1 + od)) + list(range(nd, nd + os_)):
+        s = perm[x]
+        outs = t.out_ids[t.out_off[s]:t.out_off[s + 1]].tolist()
+        oidx = x - 1 if x < nd else od + x - nd
+        payload, count = ot[oidx].tolist()
+        assert count == len(outs) and payload == (outs[0] if count == 1 else int(t.out_off[s]))
+    assert d["compact_bytes"] <= 232448 - (1024 + 32 * 2 * 512 + 512 + 256) - 1024
+    if which == "c2":
+        assert S > 15000 and d["stt_bytes"] > 1_000_000  # the dense table would not fit
+
+
 def test_classes_and_stride():
     t = ac.compile_table([b"abc", b"zz"])
     assert t.info["n_classes"] == 5  # a, b, c, z + class 0
