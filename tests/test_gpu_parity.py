@@ -104,7 +104,12 @@ def test_compact_tier(name, n, P, variant):
     stt = ac.build(w.patterns, tier=ac.TIER_COMPACT)
     assert stt.tier_name == "compact"
     want = oracle_keys(o, w.text)
-    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
+    try:
+        got = gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant)
+    except ac.AcError as e:  # a fat-ring variant cannot hold a big COMPACT table
+        assert variant != 0 and "no room" in str(e) and stt.info["compact_bytes"] > 150_000
+        return
+    assert_same(got, want)
     if variant == 0:
         assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_GLOBAL), want)
 
