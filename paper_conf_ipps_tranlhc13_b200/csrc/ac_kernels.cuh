@@ -85,17 +85,33 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
 
 // The entry delta(s, cls): next state in the low bits, output flag on top.
 // COMPACT: a dense row, or a sparse record's exception, or the dense row of
-// the record's default state fd(s) -- at most two shared-memory loads.
+// the record's default state fd(s) -- at most two shared-memory loads, issued
+// as predicated loads so lanes in dense and sparse states never diverge.
+__device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
+    const uint32_t sp = s >= st.c_dense;
+    const uint32_t ad = base + ((s * st.c_dstride + cls) << 1);
+    const uint32_t as = base + st.c_sparse_off + ((s - st.c_dense) << 3);
+    uint32_t lo = 0, hi = 0;
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t"
+        "@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t"
+        "@!p ld.shared.u16 %0, [%4];\n\t}"
+        : "+r"(lo), "+r"(hi)
+        : "r"(as), "r"(sp), "r"(ad));
+    const uint32_t h1 = ((lo >> 16) & 0xFFu) == cls, h2 = (lo >> 24) == cls;
+    const uint32_t need = sp & (1u ^ (h1 | h2));  // sparse and no exception hit
+    const uint32_t ad2 = base + (((lo & 0xFFFFu) * st.c_dstride + cls) << 1);
+    uint32_t e3 = 0;
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u16 %0, [%1];\n\t}"
+        : "+r"(e3)
+        : "r"(ad2), "r"(need));
+    const uint32_t ex = h1 ? (hi & 0xFFFFu) : (hi >> 16);
+    return sp ? (need ? e3 : ex) : lo;
+}
+
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t next_entry(const E *s_stt, const SttView &st, uint32_t s, uint32_t cls) {
     if constexpr (TIER == AC_TIER_COMPACT) {
-        const uint16_t *dense = reinterpret_cast<const uint16_t *>(s_stt);
-        if (s < st.c_dense) return dense[s * st.c_dstride + cls];
-        const uint2 r = reinterpret_cast<const uint2 *>(reinterpret_cast<const uint8_t *>(s_stt) +
-                                                        st.c_sparse_off)[s - st.c_dense];
-        if (cls == ((r.x >> 16) & 0xFFu)) return r.y & 0xFFFFu;
-        if (cls == (r.x >> 24)) return r.y >> 16;
-        return dense[(r.x & 0xFFFFu) * st.c_dstride + cls];
+        return compact_next(smem_u32(s_stt), st, s, cls);
     } else {
         return stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
     }
@@ -156,6 +172,18 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
     s = e & EntryBits<E>::MASK;
+    if constexpr (TIER == AC_TIER_COMPACT && MODE != MODE_EMIT) {
+        // branch-free count: a predicated load of the output-table count
+        const uint32_t f = (e >> 15) & (live ? 1u : 0u);
+        const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
+        const uint32_t oa = smem_u32(s_stt) + st.c_out_off + (oidx << 3) + 4;
+        uint32_t c = 0;
+        asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u32 %0, [%1];\n\t}"
+            : "+r"(c)
+            : "r"(oa), "r"(f));
+        cnt += c;
+        return;
+    }
     if ((e & EntryBits<E>::FLAG) && live) {
         const uint32_t c = out_count<E, TIER>(s_stt, st, s);
         if constexpr (MODE == MODE_EMIT) {

@@ -140,12 +140,13 @@ def test_c3_hybrid_and_global_tiers():
         assert_same(gpu_keys(stt, w.text), want)
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5])
-@pytest.mark.parametrize("name", ["c1", "c2"])
-def test_staged_variants(variant, name):
-    w = synth.make(name, n=(2 << 20) + 4321, n_patterns=None if name == "c1" else 400)
+@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7])
+@pytest.mark.parametrize("name,tier", [("c1", ac.TIER_AUTO), ("c2", ac.TIER_GLOBAL), ("c2s", ac.TIER_COMPACT)])
+def test_staged_variants(variant, name, tier):
+    P = {"c1": None, "c2": 400, "c2s": 80}[name]
+    w = synth.make(name[:2], n=(2 << 20) + 4321, n_patterns=P)
     o = Oracle(w.patterns)
-    stt = ac.build(w.patterns)
+    stt = ac.build(w.patterns, tier=tier)
     want = oracle_keys(o, w.text)
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant, chain_bytes=96), want)
