@@ -139,9 +139,15 @@ typedef struct {
     uint32_t kernel;       /* AC_KERNEL_*                                    */
     uint32_t chain_bytes;  /* bytes owned per thread chain (0 = auto; STAGED:
                               rounded to the tile width)                     */
-    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..5 (DESIGN.md
-                              "Staged variants": threads x chains/thread x
-                              tile width x ring depth)                       */
+    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..7 (DESIGN.md
+                              "Staged variants": warps x chains/lane x tile
+                              width x ring depth)                            */
+    uint32_t scratch_slots;/* list mode: records each chain may park in its
+                              scratch slot during the single emitting pass
+                              (0 = auto from cap); chains with more are
+                              re-scanned straight into place                 */
+    uint32_t two_pass;     /* list mode: 1 = count pass + emit pass instead
+                              of the single pass (ablation / fallback)       */
     uint32_t n_events;     /* pairs available in `events`                    */
     void **events;         /* optional cudaEvent_t[2 * n_events]: events[2i]
                               and events[2i+1] are recorded on the stream

@@ -67,7 +67,8 @@ class ac_stt_info(ctypes.Structure):
 
 class ac_match_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("kernel", ctypes.c_uint32), ("chain_bytes", ctypes.c_uint32),
-                ("variant", ctypes.c_uint32), ("n_events", ctypes.c_uint32),
+                ("variant", ctypes.c_uint32), ("scratch_slots", ctypes.c_uint32), ("two_pass", ctypes.c_uint32),
+                ("n_events", ctypes.c_uint32),
                 ("events", ctypes.POINTER(ctypes.c_void_p))]
 
 
@@ -193,8 +194,10 @@ def _check_text(text: torch.Tensor):
         raise ValueError("text must be 1-D and contiguous")
 
 
-def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, events=None):
-    o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, 0, None)
+def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, scratch_slots: int = 0,
+           two_pass: bool = False, events=None):
+    o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, scratch_slots,
+                      1 if two_pass else 0, 0, None)
     if events:
         arr = (ctypes.c_void_p * (2 * len(events)))(*[e.cuda_event for pair in events for e in pair])
         o.n_events = len(events)
@@ -205,10 +208,10 @@ def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, ev
 
 def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: torch.Tensor, *,
                 n_halo: int = 0, base: int = 0, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0,
-                variant: int = 0, events=None) -> int:
+                variant: int = 0, scratch_slots: int = 0, two_pass: bool = False, events=None) -> int:
     """Enqueue the scan; result (int64[2] CUDA) receives (count, status).
     ``text`` holds n_owned + n_halo bytes.  ``kernel``/``chain_bytes``/
-    ``variant`` select the scan (ac_match_opts).  ``events``: optional list
+    ``variant``/``scratch_slots``/``two_pass`` select the scan (ac_match_opts).  ``events``: optional list
     of (start, end) torch.cuda.Event pairs (already created, i.e. recorded
     once) recorded around each kernel launch.  Returns the number of kernel
     launches issued."""
@@ -226,7 +229,7 @@ def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: 
         cap = out.numel()
         # non-NULL selects list mode; with cap == 0 the status gates every write
         optr = out.data_ptr() if cap else result.data_ptr()
-    o = _mopts(kernel, chain_bytes, variant, events)
+    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events)
     L = lib()
     _check(L.ac_match_async(stt.handle, text.data_ptr() if n_total else None, n_total - n_halo, n_halo, base,
                             optr, cap, result.data_ptr(), _stream_ptr(stream), ctypes.byref(o)))

@@ -292,27 +292,66 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         so.total = reinterpret_cast<unsigned long long *>(&d_res->count);
         return scan(MODE_COUNT_TOTAL, "k_scan_global(count)", "k_scan_staged(count)");
     }
-    // --- list mode: counts | chain_end | tile_state | counter
+    // --- list mode workspace: counts | chain_end | list | tile_state | counters
+    const bool two_pass = opts && opts->two_pass;
     const size_t tiles = offsets_tiles(n_chains);
-    const size_t bytes = n_chains * 8 * 2 + tiles * 8 + 16;
+    const size_t bytes = n_chains * 8 * 3 + tiles * 8 + 16;
     void *ws = nullptr;
     AC_CUDA(cudaMallocAsync(&ws, bytes, stream), "cudaMallocAsync(workspace)");
     uint64_t *counts = static_cast<uint64_t *>(ws);
     uint64_t *chain_end = counts + n_chains;
-    uint64_t *tile_state = chain_end + n_chains;
+    uint64_t *list = chain_end + n_chains;
+    uint64_t *tile_state = list + n_chains;
     unsigned int *counter = reinterpret_cast<unsigned int *>(tile_state + tiles);
+    unsigned int *list_n = counter + 1;
     so.chain_counts = counts;
     so.chain_end = chain_end;
+    // single pass: each chain keeps its first q records in a scratch slot
+    uint64_t q = opts && opts->scratch_slots ? opts->scratch_slots : 4 * (cap / n_chains) + 64;
+    if (q > 4096) q = 4096;
+    const uint64_t max_scratch = 8ull << 30;
+    if (n_chains * q * 8 > max_scratch) q = max_scratch / (n_chains * 8);
+    if (q == 0) q = 1;
+    void *scratch = nullptr;
+    if (!two_pass) {
+        cudaError_t e = cudaMallocAsync(&scratch, n_chains * q * 8, stream);
+        if (e != cudaSuccess) {
+            cudaFreeAsync(ws, stream);
+            return cuda_fail(e, "cudaMallocAsync(scratch)");
+        }
+        so.scratch = static_cast<uint64_t *>(scratch);
+        so.q = (uint32_t)q;
+    }
     auto run = [&]() -> ac_status {
         AC_CUDA(cudaMemsetAsync(tile_state, 0, tiles * 8 + 16, stream), "memset workspace");
-        ac_status rc = scan(MODE_COUNT_CHAINS, "k_scan_global(count)", "k_scan_staged(count)");
+        if (two_pass) {
+            ac_status rc = scan(MODE_COUNT_CHAINS, "k_scan_global(count)", "k_scan_staged(count)");
+            if (rc != AC_OK) return rc;
+            pre();
+            AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream),
+                    "k_offsets");
+            post("k_offsets");
+            return scan(MODE_EMIT, "k_scan_global(emit)", "k_scan_staged(emit)");
+        }
+        ac_status rc = scan(MODE_EMIT_OPT, "k_scan_global(emit1)", "k_scan_staged(emit1)");
         if (rc != AC_OK) return rc;
         pre();
         AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream), "k_offsets");
         post("k_offsets");
-        return scan(MODE_EMIT, "k_scan_global(emit)", "k_scan_staged(emit)");
+        pre();
+        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, h->num_sms,
+                              stream),
+                "k_gather");
+        post("k_gather");
+        pre();
+        AC_CUDA(launch_rewalk(eb, tier_g, d_text, n_total, sg, ra, rb, g, so, list, list_n, smem_g, h->num_sms,
+                              stream),
+                "k_rewalk");
+        post("k_rewalk");
+        return AC_OK;
     };
     const ac_status rc = run();
+    if (scratch) cudaFreeAsync(scratch, stream);
     cudaFreeAsync(ws, stream);
     return rc;
 }

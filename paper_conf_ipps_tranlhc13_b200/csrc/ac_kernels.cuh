@@ -37,6 +37,8 @@
 // generic load), GLOBAL (L1/L2 only).
 #pragma once
 
+#include <type_traits>
+
 #include "ac_scan.cuh"
 
 namespace acx {
@@ -172,7 +174,7 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
     s = e & EntryBits<E>::MASK;
-    if constexpr (TIER == AC_TIER_COMPACT && MODE != MODE_EMIT) {
+    if constexpr (TIER == AC_TIER_COMPACT && (MODE == MODE_COUNT_TOTAL || MODE == MODE_COUNT_CHAINS)) {
         // branch-free count: a predicated load of the output-table count
         const uint32_t f = (e >> 15) & (live ? 1u : 0u);
         const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
@@ -193,6 +195,19 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                 so.out[--wp] = key0 | p;
             } else {
                 for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
+            }
+        } else if constexpr (MODE == MODE_EMIT_OPT) {
+            // wp = end of this chain's scratch slot; record k goes to wp-1-k
+            const uint64_t key0 = (so.base + pos) << 24;
+            const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
+            if (c == 1) {
+                if (cnt < so.q) so.scratch[wp - 1 - cnt] = key0 | p;
+                cnt++;
+            } else {
+                for (uint32_t j = p + c; j > p; --j) {
+                    if (cnt < so.q) so.scratch[wp - 1 - cnt] = key0 | __ldg(st.out_ids + j - 1);
+                    cnt++;
+                }
             }
         } else {
             cnt += c;
@@ -264,14 +279,49 @@ __global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ 
         const uint64_t g = r_c0 + ci;
         uint64_t wp = 0;
         if constexpr (MODE == MODE_EMIT) wp = so.chain_end[g];
+        if constexpr (MODE == MODE_EMIT_OPT) wp = (g + 1) * so.q;
         uint32_t s = 0;
         walk_global<E, TIER, MODE, false>(text, own_hi, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
         walk_global<E, TIER, MODE, true>(text, lo, own_hi, s, cnt, wp, s_cmap, s_stt, st, so);
-        if constexpr (MODE == MODE_COUNT_CHAINS) so.chain_counts[g] = cnt;
+        if constexpr (MODE == MODE_COUNT_CHAINS || MODE == MODE_EMIT_OPT) so.chain_counts[g] = cnt;
     }
     if constexpr (MODE == MODE_COUNT_TOTAL) {
         const unsigned long long tot = warp_sum(cnt);
         if ((threadIdx.x & 31) == 0 && tot) atomicAdd(so.total, tot);
+    }
+}
+
+// Re-scan the chains listed by k_gather (their matches overflowed the
+// scratch slot) in MODE_EMIT, straight into their final positions.
+template <typename E, int TIER>
+__global__ void __launch_bounds__(GT) k_rewalk(const uint8_t *__restrict__ text, uint64_t n_total, SttView st,
+                                               Region ra, Region rb, StagedGeom g, ScanOut so,
+                                               const uint64_t *__restrict__ list, const unsigned int *list_n) {
+    const uint32_t nl = *list_n;
+    if (nl == 0 || so.res->status != AC_OK) return;  // uniform: skip staging entirely
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint8_t *s_cmap = smem;
+    E *s_stt = reinterpret_cast<E *>(smem + 256);
+    stage_tables<E>(s_cmap, s_stt, st);
+    __syncthreads();
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nl; i += gridDim.x * blockDim.x) {
+        const uint64_t gi = list[i];
+        uint64_t lo, own_hi;
+        if (gi < ra.n_chains) {
+            lo = ra.lo + gi * ra.chain_len;
+            own_hi = min(lo + ra.chain_len, ra.hi);
+        } else if (g.n_chains && gi >= g.chain0 && gi < g.chain0 + g.n_chains) {
+            lo = g.m0 + (gi - g.chain0) * g.chain_len;
+            own_hi = lo + g.chain_len;
+        } else {
+            lo = rb.lo + (gi - rb.chain0) * rb.chain_len;
+            own_hi = min(lo + rb.chain_len, rb.hi);
+        }
+        const uint64_t walk_hi = min(own_hi + (uint64_t)st.halo, n_total);
+        uint64_t wp = so.chain_end[gi], cnt = 0;
+        uint32_t s = 0;
+        walk_global<E, TIER, MODE_EMIT, false>(text, own_hi, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
+        walk_global<E, TIER, MODE_EMIT, true>(text, lo, own_hi, s, cnt, wp, s_cmap, s_stt, st, so);
     }
 }
 
@@ -382,6 +432,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
         hlen[k] = (uint32_t)(rest < H ? rest : H);
         if constexpr (MODE == MODE_EMIT)
             if (live[k]) wp[k] = so.chain_end[g.chain0 + c];
+        if constexpr (MODE == MODE_EMIT_OPT) wp[k] = (g.chain0 + c + 1) * so.q;
         // the last chain's halo row is outside the tensor map (and any halo
         // wider than the next chain): warm up from global memory instead
         if (live[k] && (!tma_halo || c + 1 == g.n_chains)) {
@@ -438,7 +489,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
         if (lane == 0 && j + NST < m) issue(j + NST);
     }
 
-    if constexpr (MODE == MODE_COUNT_CHAINS) {
+    if constexpr (MODE == MODE_COUNT_CHAINS || MODE == MODE_EMIT_OPT) {
 #pragma unroll
         for (int k = 0; k < K; k++)
             if (live[k]) so.chain_counts[g.chain0 + row0 + k * 32 + lane] = cnt[k];
@@ -453,6 +504,18 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 }
 
 // ---------------------------------------------------------------- launchers
+// Dispatch a runtime scan mode to a template argument.
+template <typename F>
+static cudaError_t with_mode(int mode, F &&f) {
+    switch (mode) {
+        case MODE_COUNT_TOTAL: return f(std::integral_constant<int, MODE_COUNT_TOTAL>{});
+        case MODE_COUNT_CHAINS: return f(std::integral_constant<int, MODE_COUNT_CHAINS>{});
+        case MODE_EMIT: return f(std::integral_constant<int, MODE_EMIT>{});
+        case MODE_EMIT_OPT: return f(std::integral_constant<int, MODE_EMIT_OPT>{});
+    }
+    return cudaErrorInvalidValue;
+}
+
 template <typename E, int TIER, int MODE>
 static cudaError_t launch_global_m(const uint8_t *text, uint64_t n_total, const SttView &st, const Region &a,
                                    const Region &b, const ScanOut &so, size_t smem, cudaStream_t stream) {
@@ -473,15 +536,45 @@ cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint6
                                const Region &a, const Region &b, const ScanOut &so, size_t smem_stt,
                                cudaStream_t stream) {
     const size_t smem = 256 + smem_stt;
-    if (eb == 2) {
-        if (mode == MODE_COUNT_TOTAL) return launch_global_m<uint16_t, TIER, MODE_COUNT_TOTAL>(text, n_total, st, a, b, so, smem, stream);
-        if (mode == MODE_COUNT_CHAINS) return launch_global_m<uint16_t, TIER, MODE_COUNT_CHAINS>(text, n_total, st, a, b, so, smem, stream);
-        return launch_global_m<uint16_t, TIER, MODE_EMIT>(text, n_total, st, a, b, so, smem, stream);
+    if (eb == 2)
+        return with_mode(mode, [&](auto m) {
+            return launch_global_m<uint16_t, TIER, decltype(m)::value>(text, n_total, st, a, b, so, smem, stream);
+        });
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return cudaErrorInvalidValue;  // COMPACT is 16-bit only
+    } else {
+        return with_mode(mode, [&](auto m) {
+            return launch_global_m<uint32_t, TIER, decltype(m)::value>(text, n_total, st, a, b, so, smem, stream);
+        });
     }
-    if constexpr (TIER == AC_TIER_COMPACT) return cudaErrorInvalidValue;  // COMPACT is 16-bit only
-    if (mode == MODE_COUNT_TOTAL) return launch_global_m<uint32_t, TIER, MODE_COUNT_TOTAL>(text, n_total, st, a, b, so, smem, stream);
-    if (mode == MODE_COUNT_CHAINS) return launch_global_m<uint32_t, TIER, MODE_COUNT_CHAINS>(text, n_total, st, a, b, so, smem, stream);
-    return launch_global_m<uint32_t, TIER, MODE_EMIT>(text, n_total, st, a, b, so, smem, stream);
+}
+
+template <typename E, int TIER>
+static cudaError_t launch_rewalk_e(const uint8_t *text, uint64_t n_total, const SttView &st, const Region &a,
+                                   const Region &b, const StagedGeom &g, const ScanOut &so, const uint64_t *list,
+                                   const unsigned int *list_n, size_t smem, int num_sms, cudaStream_t stream) {
+    auto kern = k_rewalk<E, TIER>;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    kern<<<num_sms, GT, smem, stream>>>(text, n_total, st, a, b, g, so, list, list_n);
+    return cudaGetLastError();
+}
+
+template <int TIER>
+cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_total, const SttView &st,
+                               const Region &a, const Region &b, const StagedGeom &g, const ScanOut &so,
+                               const uint64_t *list, const unsigned int *list_n, size_t smem_stt, int num_sms,
+                               cudaStream_t stream) {
+    const size_t smem = 256 + smem_stt;
+    if (eb == 2)
+        return launch_rewalk_e<uint16_t, TIER>(text, n_total, st, a, b, g, so, list, list_n, smem, num_sms, stream);
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return cudaErrorInvalidValue;
+    } else {
+        return launch_rewalk_e<uint32_t, TIER>(text, n_total, st, a, b, g, so, list, list_n, smem, num_sms, stream);
+    }
 }
 
 template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST>
@@ -515,15 +608,19 @@ template <int TIER>
 cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtensorMap &tmap, const uint8_t *mtext,
                                const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
                                cudaStream_t stream) {
-    if (eb == 2) {
-        if (mode == MODE_COUNT_TOTAL) return launch_staged_m<uint16_t, TIER, MODE_COUNT_TOTAL>(variant, tmap, mtext, st, g, so, smem_stt, stream);
-        if (mode == MODE_COUNT_CHAINS) return launch_staged_m<uint16_t, TIER, MODE_COUNT_CHAINS>(variant, tmap, mtext, st, g, so, smem_stt, stream);
-        return launch_staged_m<uint16_t, TIER, MODE_EMIT>(variant, tmap, mtext, st, g, so, smem_stt, stream);
+    if (eb == 2)
+        return with_mode(mode, [&](auto m) {
+            return launch_staged_m<uint16_t, TIER, decltype(m)::value>(variant, tmap, mtext, st, g, so, smem_stt,
+                                                                       stream);
+        });
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return cudaErrorInvalidValue;  // COMPACT is 16-bit only
+    } else {
+        return with_mode(mode, [&](auto m) {
+            return launch_staged_m<uint32_t, TIER, decltype(m)::value>(variant, tmap, mtext, st, g, so, smem_stt,
+                                                                       stream);
+        });
     }
-    if constexpr (TIER == AC_TIER_COMPACT) return cudaErrorInvalidValue;  // COMPACT is 16-bit only
-    if (mode == MODE_COUNT_TOTAL) return launch_staged_m<uint32_t, TIER, MODE_COUNT_TOTAL>(variant, tmap, mtext, st, g, so, smem_stt, stream);
-    if (mode == MODE_COUNT_CHAINS) return launch_staged_m<uint32_t, TIER, MODE_COUNT_CHAINS>(variant, tmap, mtext, st, g, so, smem_stt, stream);
-    return launch_staged_m<uint32_t, TIER, MODE_EMIT>(variant, tmap, mtext, st, g, so, smem_stt, stream);
 }
 
 }  // namespace acx

@@ -120,6 +120,53 @@ __global__ void __launch_bounds__(OT) k_offsets(const uint64_t *__restrict__ cou
 
 size_t offsets_tiles(uint64_t n) { return (size_t)((n + OTILE - 1) / OTILE); }
 
+// ------------------------------------------------------------- k_gather
+// One warp per chain (grid-stride): a chain whose count fits its scratch slot
+// is copied, coalesced, from the tail of the slot to [chain_end - cnt,
+// chain_end); an overflowed chain is appended to the re-walk list.
+__global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ counts,
+                                                const uint64_t *__restrict__ chain_end, uint64_t n_chains,
+                                                const uint64_t *__restrict__ scratch, uint32_t q,
+                                                uint64_t *__restrict__ out, const ac_result *res, uint64_t *list,
+                                                unsigned int *list_n) {
+    if (res->status != AC_OK) return;
+    const int lane = threadIdx.x & 31;
+    const uint64_t warps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+    for (uint64_t c = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < n_chains; c += warps) {
+        const uint64_t cnt = counts[c];
+        if (cnt == 0) continue;
+        if (cnt > q) {
+            if (lane == 0) list[atomicAdd(list_n, 1u)] = c;
+            continue;
+        }
+        const uint64_t *src = scratch + c * q + (q - cnt);
+        uint64_t *dst = out + chain_end[c] - cnt;
+        for (uint64_t i = lane; i < cnt; i += 32) dst[i] = __ldg(src + i);
+    }
+}
+
+cudaError_t launch_gather(const uint64_t *counts, const uint64_t *chain_end, uint64_t n_chains,
+                          const uint64_t *scratch, uint32_t q, uint64_t *out, const ac_result *res, uint64_t *list,
+                          unsigned int *list_n, int num_sms, cudaStream_t stream) {
+    if (n_chains == 0) return cudaSuccess;
+    const uint64_t want = (n_chains + 7) / 8;
+    const unsigned grid = (unsigned)(want < (uint64_t)num_sms * 8 ? want : (uint64_t)num_sms * 8);
+    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_rewalk(uint32_t eb, uint32_t tier, const uint8_t *text, uint64_t n_total, const SttView &st,
+                          const Region &a, const Region &b, const StagedGeom &g, const ScanOut &so,
+                          const uint64_t *list, const unsigned int *list_n, size_t smem_stt, int num_sms,
+                          cudaStream_t stream) {
+    switch (tier) {
+        case AC_TIER_SMEM: return launch_rewalk_tier<AC_TIER_SMEM>(eb, text, n_total, st, a, b, g, so, list, list_n, smem_stt, num_sms, stream);
+        case AC_TIER_HYBRID: return launch_rewalk_tier<AC_TIER_HYBRID>(eb, text, n_total, st, a, b, g, so, list, list_n, smem_stt, num_sms, stream);
+        case AC_TIER_COMPACT: return launch_rewalk_tier<AC_TIER_COMPACT>(eb, text, n_total, st, a, b, g, so, list, list_n, smem_stt, num_sms, stream);
+        default: return launch_rewalk_tier<AC_TIER_GLOBAL>(eb, text, n_total, st, a, b, g, so, list, list_n, smem_stt, num_sms, stream);
+    }
+}
+
 cudaError_t launch_offsets(const uint64_t *counts, uint64_t n, uint64_t *chain_end, uint64_t *tile_state,
                            unsigned int *tile_counter, ac_result *res, uint64_t cap, int emitting,
                            cudaStream_t stream) {

@@ -10,7 +10,11 @@
 
 namespace acx {
 
-enum ScanMode { MODE_COUNT_TOTAL = 0, MODE_COUNT_CHAINS = 1, MODE_EMIT = 2 };
+// COUNT_TOTAL: count only (atomic total).  COUNT_CHAINS: per-chain counts.
+// EMIT: write records at known chain end offsets (second pass).
+// EMIT_OPT: one pass -- per-chain counts AND the chain's first q records
+// written into its scratch slot; k_gather moves them to their final place.
+enum ScanMode { MODE_COUNT_TOTAL = 0, MODE_COUNT_CHAINS = 1, MODE_EMIT = 2, MODE_EMIT_OPT = 3 };
 
 // Read-only automaton as the kernels see it.
 struct SttView {
@@ -44,6 +48,8 @@ struct ScanOut {
     const ac_result *res;           // MODE_EMIT: skip writing when res->status != AC_OK
     uint64_t *out;                  // MODE_EMIT: records
     uint64_t base;                  // global position of shard byte 0
+    uint64_t *scratch;              // MODE_EMIT_OPT: q slots per chain
+    uint32_t q;
 };
 
 // Geometry of the TMA-staged main region.
@@ -85,6 +91,17 @@ cudaError_t launch_offsets(const uint64_t *counts, uint64_t n, uint64_t *chain_e
 
 size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
 
+// Single-pass list mode helpers: k_gather copies every chain's scratch slot
+// to its final position (or lists the chain when it overflowed); k_rewalk
+// re-scans the listed chains in MODE_EMIT.
+cudaError_t launch_gather(const uint64_t *counts, const uint64_t *chain_end, uint64_t n_chains,
+                          const uint64_t *scratch, uint32_t q, uint64_t *out, const ac_result *res,
+                          uint64_t *list, unsigned int *list_n, int num_sms, cudaStream_t stream);
+cudaError_t launch_rewalk(uint32_t entry_bytes, uint32_t tier, const uint8_t *text, uint64_t n_total,
+                          const SttView &st, const Region &a, const Region &b, const StagedGeom &g,
+                          const ScanOut &so, const uint64_t *list, const unsigned int *list_n, size_t smem_stt,
+                          int num_sms, cudaStream_t stream);
+
 // per-tier instantiations (ac_tier_*.cu)
 template <int TIER>
 cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint64_t n_total, const SttView &st,
@@ -93,6 +110,11 @@ cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint6
 template <int TIER>
 cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtensorMap &tmap, const uint8_t *mtext,
                                const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
+                               cudaStream_t stream);
+template <int TIER>
+cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_total, const SttView &st,
+                               const Region &a, const Region &b, const StagedGeom &g, const ScanOut &so,
+                               const uint64_t *list, const unsigned int *list_n, size_t smem_stt, int num_sms,
                                cudaStream_t stream);
 int staged_variant_count();
 const StagedConfig &staged_variant(int v);  // v in [1, staged_variant_count()]

@@ -9,3 +9,10 @@ template cudaError_t launch_staged_tier<AC_TIER_HYBRID>(int, uint32_t, int, cons
                                                      const SttView &, const StagedGeom &, const ScanOut &, size_t,
                                                      cudaStream_t);
 }  // namespace acx
+
+namespace acx {
+template cudaError_t launch_rewalk_tier<AC_TIER_HYBRID>(uint32_t, const uint8_t *, uint64_t, const SttView &,
+                                                     const Region &, const Region &, const StagedGeom &,
+                                                     const ScanOut &, const uint64_t *, const unsigned int *, size_t,
+                                                     int, cudaStream_t);
+}  // namespace acx

@@ -39,6 +39,10 @@ def gpu_keys(stt, text_np: np.ndarray, **kw) -> np.ndarray:
     t = torch.from_numpy(np.ascontiguousarray(text_np)).cuda() if text_np.size else torch.empty(0, dtype=torch.uint8, device="cuda")
     c, recs = ac.match(stt, t, **kw)
     cnt = ac.count(stt, t, **{k: v for k, v in kw.items() if k in ("kernel", "chain_bytes", "variant")})
+    if c:  # the two-pass list mode and a forced-overflow single pass agree bit for bit
+        _, r2 = ac.match(stt, t, two_pass=True, **kw)
+        _, r3 = ac.match(stt, t, scratch_slots=2, **kw)  # most chains overflow -> k_rewalk
+        assert torch.equal(r2, recs) and torch.equal(r3, recs)
     assert cnt == c
     return recs.cpu().numpy()
 
@@ -303,6 +307,30 @@ def test_shard_api_concatenation():
             c, recs = ac.match(stt, t[lo:hi + halo], n_halo=halo, base=lo)
             parts.append(recs.cpu().numpy())
         assert_same(np.concatenate(parts), want)
+
+
+def test_match_sharded_nccl_world1():
+    import os
+    import socket
+    import torch.distributed as dist
+    from paper_conf_ipps_tranlhc13_b200.dist import match_sharded, plan_shards
+    w = synth.make("c2", n=(1 << 20) + 3, n_patterns=200)
+    o = Oracle(w.patterns)
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        stt = ac.build(w.patterns)
+        (sh,) = plan_shards(w.text.size, 1, stt.maxlen)
+        t = torch.from_numpy(w.text[sh.lo:sh.read_hi]).cuda()
+        total, recs = match_sharded(stt, t, sh, gather=True)
+        want = oracle_keys(o, w.text)
+        assert total == want.size
+        assert_same(recs.cpu().numpy(), want)
+    finally:
+        dist.destroy_process_group()
 
 
 def test_host_entry_point():
