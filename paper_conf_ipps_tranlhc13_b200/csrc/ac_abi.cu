@@ -56,6 +56,34 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     return fn;
 }
 
+// Per-thread, per-device side stream + fork/join events (created lazily,
+// kept for the thread's lifetime).
+struct SideStream {
+    cudaStream_t stream = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+};
+
+static ac_status side_stream(int device, SideStream **out) {
+    static thread_local SideStream per_dev[64];
+    if (device < 0 || device >= 64) {
+        set_error("device index out of range");
+        return AC_ERR_INVALID_ARG;
+    }
+    SideStream &s = per_dev[device];
+    if (!s.stream) {
+        int prev = -1;
+        cudaGetDevice(&prev);
+        AC_CUDA(cudaSetDevice(device), "cudaSetDevice");
+        cudaError_t e = cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming);
+        if (prev >= 0) cudaSetDevice(prev);
+        if (e != cudaSuccess) return cuda_fail(e, "side stream setup");
+    }
+    *out = &s;
+    return AC_OK;
+}
+
 static void keep_pool(int device) {
     static std::mutex mu;
     static bool done[64] = {false};
@@ -274,11 +302,26 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     so.base = base;
     so.res = d_res;
     so.out = reinterpret_cast<uint64_t *>(d_out);
+    // The few head/tail chains (global kernel) are latency bound: when a
+    // staged main region exists they run concurrently on a side stream
+    // (event fork/join, capturable in a CUDA graph).
+    SideStream *side = nullptr;
+    if (any_global && g.n_chains) {
+        ac_status rc = side_stream(h->device, &side);
+        if (rc != AC_OK) return rc;
+    }
     auto scan = [&](int mode, const char *gname, const char *sname) -> ac_status {
         if (any_global) {
+            cudaStream_t gs = stream;
+            if (side) {
+                AC_CUDA(cudaEventRecord(side->fork, stream), "cudaEventRecord(fork)");
+                AC_CUDA(cudaStreamWaitEvent(side->stream, side->fork, 0), "cudaStreamWaitEvent(fork)");
+                gs = side->stream;
+            }
             pre();
-            AC_CUDA(launch_scan_global(mode, eb, tier_g, d_text, n_total, sg, ra, rb, so, smem_g, stream), gname);
+            AC_CUDA(launch_scan_global(mode, eb, tier_g, d_text, n_total, sg, ra, rb, so, smem_g, gs), gname);
             post(gname);
+            if (side) AC_CUDA(cudaEventRecord(side->join, side->stream), "cudaEventRecord(join)");
         }
         if (g.n_chains) {
             pre();
@@ -286,6 +329,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
                     sname);
             post(sname);
         }
+        if (side) AC_CUDA(cudaStreamWaitEvent(stream, side->join, 0), "cudaStreamWaitEvent(join)");
         return AC_OK;
     };
     if (!emit) {
