@@ -167,6 +167,71 @@ __device__ __forceinline__ uint32_t out_payload(const E *s_stt, const SttView &s
     }
 }
 
+// (payload, count) of state s if f != 0, else (0, 0) -- predicated loads
+// through the state's residency tier, so lanes never branch on a match.
+template <typename E, int TIER, bool PAYLOAD>
+__device__ __forceinline__ uint2 out_info_pred(const E *s_stt, const SttView &st, uint32_t s, uint32_t f) {
+    uint32_t pay = 0, c = 0;
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
+        const uint32_t a = smem_u32(s_stt) + st.c_out_off + (oidx << 3);
+        asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t}"
+            : "+r"(pay), "+r"(c)
+            : "r"(a), "r"(f));
+    } else {
+        const uint32_t ip = s * st.stride + st.info_col;            // payload (u32, 4-byte aligned)
+        const uint32_t ic = ip + (sizeof(E) == 2 ? 2 : 1);           // count (E)
+        if constexpr (TIER == AC_TIER_SMEM) {
+            const uint32_t b = smem_u32(s_stt);
+            if constexpr (sizeof(E) == 2)
+                asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u16 %0, [%1];\n\t}"
+                    : "+r"(c)
+                    : "r"(b + ic * 2), "r"(f));
+            else
+                asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u32 %0, [%1];\n\t}"
+                    : "+r"(c)
+                    : "r"(b + ic * 4), "r"(f));
+            if constexpr (PAYLOAD)
+                asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u32 %0, [%1];\n\t}"
+                    : "+r"(pay)
+                    : "r"(b + ip * (uint32_t)sizeof(E)), "r"(f));
+        } else {
+            // GLOBAL: read-only global path; HYBRID: generic address (smem prefix or global)
+            const E *g = static_cast<const E *>(st.stt);
+            const E *base = (TIER == AC_TIER_HYBRID && s < st.smem_rows) ? s_stt : g;
+            const uint64_t pc = reinterpret_cast<uint64_t>(base + ic), pp = reinterpret_cast<uint64_t>(base + ip);
+            if constexpr (TIER == AC_TIER_GLOBAL) {
+                if constexpr (sizeof(E) == 2)
+                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u16 %0, [%1];\n\t}"
+                        : "+r"(c)
+                        : "l"(pc), "r"(f));
+                else
+                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u32 %0, [%1];\n\t}"
+                        : "+r"(c)
+                        : "l"(pc), "r"(f));
+                if constexpr (PAYLOAD)
+                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u32 %0, [%1];\n\t}"
+                        : "+r"(pay)
+                        : "l"(pp), "r"(f));
+            } else {
+                if constexpr (sizeof(E) == 2)
+                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.u16 %0, [%1];\n\t}"
+                        : "+r"(c)
+                        : "l"(pc), "r"(f));
+                else
+                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.u32 %0, [%1];\n\t}"
+                        : "+r"(c)
+                        : "l"(pc), "r"(f));
+                if constexpr (PAYLOAD)
+                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.u32 %0, [%1];\n\t}"
+                        : "+r"(pay)
+                        : "l"(pp), "r"(f));
+            }
+        }
+    }
+    return make_uint2(pay, c);
+}
+
 // One transition inside the owned chunk: count or emit output(s) at pos.
 template <typename E, int TIER, int MODE>
 __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp, uint32_t byte, uint64_t pos,
@@ -174,16 +239,34 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
     s = e & EntryBits<E>::MASK;
-    if constexpr (TIER == AC_TIER_COMPACT && (MODE == MODE_COUNT_TOTAL || MODE == MODE_COUNT_CHAINS)) {
-        // branch-free count: a predicated load of the output-table count
-        const uint32_t f = (e >> 15) & (live ? 1u : 0u);
-        const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
-        const uint32_t oa = smem_u32(s_stt) + st.c_out_off + (oidx << 3) + 4;
-        uint32_t c = 0;
-        asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u32 %0, [%1];\n\t}"
-            : "+r"(c)
-            : "r"(oa), "r"(f));
-        cnt += c;
+    if constexpr (MODE != MODE_EMIT) {
+        // Branch-free for the common cases: predicated loads of the output
+        // summary and a predicated store of a single-output match; only
+        // multi-output states (and saturated counts) take a branch.
+        const uint32_t f = ((e & EntryBits<E>::FLAG) != 0) & (live ? 1u : 0u);
+        const uint2 o = out_info_pred<E, TIER, MODE == MODE_EMIT_OPT>(s_stt, st, s, f);
+        uint32_t c = o.y;
+        if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
+            c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);
+        if constexpr (MODE == MODE_EMIT_OPT) {
+            // wp = end of this chain's scratch slot; record k goes to wp-1-k
+            const uint64_t key0 = (so.base + pos) << 24;
+            const uint32_t one = (c == 1u) & (cnt < so.q ? 1u : 0u);
+            uint64_t *dst = so.scratch + (wp - 1 - cnt);
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}" ::"l"(dst),
+                         "l"(key0 | o.x), "r"(one)
+                         : "memory");
+            if (c > 1u) {
+                for (uint32_t j = o.x + c; j > o.x; --j) {
+                    if (cnt < so.q) so.scratch[wp - 1 - cnt] = key0 | __ldg(st.out_ids + j - 1);
+                    cnt++;
+                }
+            } else {
+                cnt += c;
+            }
+        } else {
+            cnt += c;
+        }
         return;
     }
     if ((e & EntryBits<E>::FLAG) && live) {
