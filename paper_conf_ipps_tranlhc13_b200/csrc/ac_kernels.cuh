@@ -239,7 +239,10 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
     s = e & EntryBits<E>::MASK;
-    if constexpr (MODE != MODE_EMIT) {
+    // Counting with the dense tiers keeps the branch (flags are rare there and
+    // predicated loads cost issue slots on every byte: measured 25 % on C1).
+    constexpr bool kPred = MODE == MODE_EMIT_OPT || (TIER == AC_TIER_COMPACT && MODE != MODE_EMIT);
+    if constexpr (kPred) {
         // Branch-free for the common cases: predicated loads of the output
         // summary and a predicated store of a single-output match; only
         // multi-output states (and saturated counts) take a branch.
@@ -375,7 +378,10 @@ __global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ 
 }
 
 // Re-scan the chains listed by k_gather (their matches overflowed the
-// scratch slot) in MODE_EMIT, straight into their final positions.
+// scratch slot) straight into their final positions.  One CTA per listed
+// chain: the chain is split into GT sub-chains (each with its own halo
+// warm-up, P:163-164 again one level down), counted, block-scanned and
+// emitted -- so a dense chain costs ~2 x (L/GT + halo) steps, not L.
 template <typename E, int TIER>
 __global__ void __launch_bounds__(GT) k_rewalk(const uint8_t *__restrict__ text, uint64_t n_total, SttView st,
                                                Region ra, Region rb, StagedGeom g, ScanOut so,
@@ -383,11 +389,13 @@ __global__ void __launch_bounds__(GT) k_rewalk(const uint8_t *__restrict__ text,
     const uint32_t nl = *list_n;
     if (nl == 0 || so.res->status != AC_OK) return;  // uniform: skip staging entirely
     extern __shared__ __align__(16) uint8_t smem[];
+    __shared__ unsigned long long s_warp[GT / 32];
     uint8_t *s_cmap = smem;
     E *s_stt = reinterpret_cast<E *>(smem + 256);
     stage_tables<E>(s_cmap, s_stt, st);
     __syncthreads();
-    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nl; i += gridDim.x * blockDim.x) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (uint32_t i = blockIdx.x; i < nl; i += gridDim.x) {
         const uint64_t gi = list[i];
         uint64_t lo, own_hi;
         if (gi < ra.n_chains) {
@@ -400,11 +408,32 @@ __global__ void __launch_bounds__(GT) k_rewalk(const uint8_t *__restrict__ text,
             lo = rb.lo + (gi - rb.chain0) * rb.chain_len;
             own_hi = min(lo + rb.chain_len, rb.hi);
         }
-        const uint64_t walk_hi = min(own_hi + (uint64_t)st.halo, n_total);
-        uint64_t wp = so.chain_end[gi], cnt = 0;
+        const uint64_t sub = (own_hi - lo + GT - 1) / GT;
+        const uint64_t a = min(lo + threadIdx.x * sub, own_hi), b = min(a + sub, own_hi);
+        const uint64_t walk_hi = min(b + (uint64_t)st.halo, n_total);
+        uint64_t cnt = 0, wp = 0;
         uint32_t s = 0;
-        walk_global<E, TIER, MODE_EMIT, false>(text, own_hi, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
-        walk_global<E, TIER, MODE_EMIT, true>(text, lo, own_hi, s, cnt, wp, s_cmap, s_stt, st, so);
+        if (a < b) {
+            walk_global<E, TIER, MODE_COUNT_CHAINS, false>(text, b, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
+            walk_global<E, TIER, MODE_COUNT_CHAINS, true>(text, a, b, s, cnt, wp, s_cmap, s_stt, st, so);
+        }
+        // suffix sum: records of later sub-chains come later in canonical order
+        unsigned long long incl = cnt;
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long y = __shfl_down_sync(0xffffffffu, incl, o);
+            if (lane + o < 32) incl += y;
+        }
+        if (lane == 0) s_warp[w] = incl;
+        __syncthreads();
+        unsigned long long after = incl - cnt;
+        for (int j = w + 1; j < GT / 32; j++) after += s_warp[j];
+        __syncthreads();
+        if (a < b && cnt) {
+            wp = so.chain_end[gi] - after;
+            s = 0;
+            walk_global<E, TIER, MODE_EMIT, false>(text, b, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
+            walk_global<E, TIER, MODE_EMIT, true>(text, a, b, s, cnt, wp, s_cmap, s_stt, st, so);
+        }
     }
 }
 
