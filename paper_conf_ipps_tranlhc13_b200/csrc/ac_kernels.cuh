@@ -239,9 +239,11 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
     s = e & EntryBits<E>::MASK;
-    // Counting with the dense tiers keeps the branch (flags are rare there and
-    // predicated loads cost issue slots on every byte: measured 25 % on C1).
-    constexpr bool kPred = MODE == MODE_EMIT_OPT || (TIER == AC_TIER_COMPACT && MODE != MODE_EMIT);
+    // Predication pays where matches are dense (C2-like dictionaries, which are
+    // what land in COMPACT); with rare flags (C1/C3/C4) the predicated loads
+    // and store cost issue slots on every byte (measured: C1 list 2.6x slower),
+    // so the dense tiers keep the branch.
+    constexpr bool kPred = TIER == AC_TIER_COMPACT && MODE != MODE_EMIT;
     if constexpr (kPred) {
         // Branch-free for the common cases: predicated loads of the output
         // summary and a predicated store of a single-output match; only
