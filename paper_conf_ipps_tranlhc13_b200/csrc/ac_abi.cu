@@ -4,6 +4,7 @@
 // Phase split follows the paper: the STT is built once on the host and
 // copied to the device; the text is device resident before the scan
 // (P:148); build and copies are outside the timed scan.
+#include <algorithm>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -214,6 +215,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     if (n_owned == 0 || h->host.n_patterns == 0) return AC_OK;
 
     const uint32_t eb = h->host.entry_bytes;
+    // chain counters are 32-bit in the kernels: chain bytes x max|output| < 2^31
+    const uint64_t count_lim = h->host.max_out ? (1ull << 31) / h->host.max_out : UINT64_MAX;
     const uint64_t req_chain = opts ? opts->chain_bytes : 0;
     if (kernel == AC_KERNEL_AUTO) kernel = n_owned >= kStagedMinBytes ? AC_KERNEL_STAGED : AC_KERNEL_GLOBAL;
     int variant = opts ? (int)opts->variant : 0;
@@ -253,6 +256,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             if (L < kStagedMinChain) L = kStagedMinChain;
         }
         if (L > (1ull << 30)) L = (1ull << 30) / W * W;
+        if (L > count_lim) L = std::max<uint64_t>(W, count_lim / W * W);
         uint64_t n_main = avail / L;
         if (n_main > (1ull << 31) - R) n_main = ((1ull << 31) - R);
         ra = Region{0, head, kGlobalTailChain, (head + kGlobalTailChain - 1) / kGlobalTailChain, 0};
@@ -271,7 +275,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             cuuint64_t strides[1] = {(cuuint64_t)L};
             cuuint32_t box[2] = {(cuuint32_t)W, (cuuint32_t)(32 * cfg.k)};
             cuuint32_t estr[2] = {1, 1};
-            const CUtensorMapSwizzle swz = W == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+            const CUtensorMapSwizzle swz = !cfg.swizzle ? CU_TENSOR_MAP_SWIZZLE_NONE
+                                           : W == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
                                            : W == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
                                            : W == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
                                                      : CU_TENSOR_MAP_SWIZZLE_NONE;
@@ -292,6 +297,9 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             L = (n_owned + (uint64_t)h->num_sms * 1024 - 1) / ((uint64_t)h->num_sms * 1024);
             L = (L + 15) / 16 * 16;
             if (L < 64) L = 64;
+        }
+        if (L > count_lim) {
+            L = std::max<uint64_t>(1, count_lim);
         }
         ra = Region{0, n_owned, L, (n_owned + L - 1) / L, 0};
     }
@@ -408,6 +416,140 @@ static ac_status finish_sync(ac_result *d_res, uint64_t *count, cudaStream_t str
     if (hres.status != AC_OK) {
         set_error("match list longer than cap (" + std::to_string(hres.count) + " records needed)");
         return (ac_status)hres.status;
+    }
+    return AC_OK;
+}
+
+// ------------------------------------------------- host-buffer pipeline
+// the text is cut into chunks (shards with halos, the
+// same ownership rule as a1); H2D of chunk i+2 (copy stream) overlaps the
+// scan of chunk i (caller stream) and the D2H of chunk i-1's records (second
+// copy stream).  Each chunk's list lands at the running offset, so the host
+// list is the global canonical list.
+struct HostPipe {
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t loaded[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr}, done[2] = {nullptr, nullptr};
+    ac_result *pinned = nullptr;  // kMaxChunks results
+};
+static const uint64_t kMaxChunks = 4096, kChunk = 32ull << 20;
+
+static ac_status host_pipe(int device, HostPipe **out) {
+    static thread_local HostPipe per_dev[64];
+    if (device < 0 || device >= 64) {
+        set_error("device index out of range");
+        return AC_ERR_INVALID_ARG;
+    }
+    HostPipe &p = per_dev[device];
+    if (!p.h2d) {
+        cudaError_t e = cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p.d2h, cudaStreamNonBlocking);
+        for (int i = 0; i < 2 && e == cudaSuccess; i++) {
+            e = cudaEventCreateWithFlags(&p.loaded[i], cudaEventDisableTiming);
+            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p.freed[i], cudaEventDisableTiming);
+            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p.done[i], cudaEventDisableTiming);
+        }
+        if (e == cudaSuccess) e = cudaHostAlloc(&p.pinned, kMaxChunks * sizeof(ac_result), cudaHostAllocDefault);
+        if (e != cudaSuccess) {
+            p.h2d = nullptr;
+            return cuda_fail(e, "host pipeline setup");
+        }
+    }
+    *out = &p;
+    return AC_OK;
+}
+
+static ac_status match_host_pipelined(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac_match_t *h_out,
+                                      uint64_t cap, uint64_t *count, cudaStream_t s) {
+    int prev = -1;
+    cudaGetDevice(&prev);
+    AC_CUDA(cudaSetDevice(stt->device), "cudaSetDevice");
+    struct Restore {
+        int d;
+        ~Restore() {
+            if (d >= 0) cudaSetDevice(d);
+        }
+    } restore{prev};
+    HostPipe *P = nullptr;
+    ac_status rc = host_pipe(stt->device, &P);
+    if (rc != AC_OK) return rc;
+    const uint64_t H = stt->host.maxlen ? stt->host.maxlen - 1 : 0;
+    uint64_t CH = kChunk;
+    if (n / CH + 1 > kMaxChunks) CH = (n / (kMaxChunks - 1) + 16) / 16 * 16;
+    const uint64_t nch = n ? (n + CH - 1) / CH : 1;
+    const bool emit = h_out != nullptr;
+    uint8_t *tb[2] = {nullptr, nullptr};
+    ac_match_t *d_out = nullptr;
+    ac_result *d_res = nullptr;
+    auto cleanup = [&]() {
+        for (auto &b : tb)
+            if (b) cudaFreeAsync(b, s);
+        if (d_out) cudaFreeAsync(d_out, s);
+        if (d_res) cudaFreeAsync(d_res, s);
+        cudaStreamSynchronize(P->d2h);
+        cudaStreamSynchronize(P->h2d);
+        cudaStreamSynchronize(s);
+    };
+    cudaError_t e = cudaMallocAsync(&d_res, nch * sizeof(ac_result), s);
+    for (int b = 0; b < 2 && e == cudaSuccess && n; b++) e = cudaMallocAsync(&tb[b], CH + H + 16, s);
+    if (e == cudaSuccess && emit) e = cudaMallocAsync(&d_out, (cap ? cap : 1) * sizeof(ac_match_t), s);
+    // the copy streams must see the allocations
+    if (e == cudaSuccess) e = cudaEventRecord(P->freed[0], s);
+    if (e == cudaSuccess) e = cudaEventRecord(P->freed[1], s);
+    if (e != cudaSuccess) {
+        cleanup();
+        return cuda_fail(e, "host pipeline buffers");
+    }
+    auto lo_of = [&](uint64_t i) { return i * CH; };
+    auto own_of = [&](uint64_t i) { return std::min(CH, n - lo_of(i)); };
+    auto halo_of = [&](uint64_t i) { return std::min(H, n - lo_of(i) - own_of(i)); };
+    auto issue_h2d = [&](uint64_t j) -> cudaError_t {
+        const int b = (int)(j & 1);
+        cudaError_t err = cudaStreamWaitEvent(P->h2d, P->freed[b], 0);
+        if (err == cudaSuccess)
+            err = cudaMemcpyAsync(tb[b], h_text + lo_of(j), own_of(j) + halo_of(j), cudaMemcpyHostToDevice, P->h2d);
+        if (err == cudaSuccess) err = cudaEventRecord(P->loaded[b], P->h2d);
+        return err;
+    };
+    uint64_t off = 0;
+    bool over = false;
+    auto collect = [&](uint64_t i) -> ac_status {  // chunk i's count is needed on the host
+        AC_CUDA(cudaEventSynchronize(P->done[i & 1]), "cudaEventSynchronize");
+        const ac_result r = P->pinned[i];
+        if (r.status == AC_ERR_CAPACITY) over = true;
+        if (emit && !over && r.count)
+            AC_CUDA(cudaMemcpyAsync(h_out + off, d_out + off, r.count * sizeof(ac_match_t), cudaMemcpyDeviceToHost,
+                                    P->d2h),
+                    "D2H matches");
+        off += r.count;
+        if (emit && off > cap) over = true;
+        return AC_OK;
+    };
+    if (n) {
+        for (uint64_t j = 0; j < 2 && j < nch; j++) AC_CUDA(issue_h2d(j), "H2D text");
+    }
+    for (uint64_t i = 0; i < nch; i++) {
+        if (i > 0) {
+            rc = collect(i - 1);
+            if (rc != AC_OK) break;
+        }
+        const int b = (int)(i & 1);
+        if (n) AC_CUDA(cudaStreamWaitEvent(s, P->loaded[b], 0), "cudaStreamWaitEvent");
+        ac_match_t *dst = (emit && !over) ? d_out + off : nullptr;
+        rc = ac_match_async(stt, n ? tb[b] : nullptr, n ? own_of(i) : 0, n ? halo_of(i) : 0, lo_of(i), dst,
+                            (emit && !over) ? cap - off : 0, d_res + i, s, nullptr);
+        if (rc != AC_OK) break;
+        AC_CUDA(cudaEventRecord(P->freed[b], s), "cudaEventRecord");
+        AC_CUDA(cudaMemcpyAsync(&P->pinned[i], d_res + i, sizeof(ac_result), cudaMemcpyDeviceToHost, s), "D2H result");
+        AC_CUDA(cudaEventRecord(P->done[b], s), "cudaEventRecord");
+        if (n && i + 2 < nch) AC_CUDA(issue_h2d(i + 2), "H2D text");
+    }
+    if (rc == AC_OK) rc = collect(nch - 1);
+    cleanup();
+    if (rc != AC_OK) return rc;
+    if (count) *count = off;
+    if (emit && (over || off > cap)) {
+        set_error("match list longer than cap (" + std::to_string(off) + " records needed)");
+        return AC_ERR_CAPACITY;
     }
     return AC_OK;
 }
@@ -699,40 +841,12 @@ ac_status ac_match_host(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac
         set_error("NULL stt or text");
         return AC_ERR_INVALID_ARG;
     }
-    cudaStream_t s = static_cast<cudaStream_t>(stream);
-    uint8_t *d_text = nullptr;
-    ac_match_t *d_out = nullptr;
-    ac_result *d_res = nullptr;
-    ac_status rc = AC_OK;
-    auto cleanup = [&]() {
-        if (d_text) cudaFreeAsync(d_text, s);
-        if (d_out) cudaFreeAsync(d_out, s);
-        if (d_res) cudaFreeAsync(d_res, s);
-        cudaStreamSynchronize(s);
-    };
-    cudaError_t e;
-    if ((e = cudaMallocAsync(&d_res, sizeof(ac_result), s)) != cudaSuccess) { cleanup(); return cuda_fail(e, "alloc result"); }
-    if (n && (e = cudaMallocAsync(&d_text, n, s)) != cudaSuccess) { cleanup(); return cuda_fail(e, "alloc text"); }
-    if (h_out && cap && (e = cudaMallocAsync(&d_out, cap * sizeof(ac_match_t), s)) != cudaSuccess) {
-        cleanup();
-        return cuda_fail(e, "alloc out");
+    try {
+        return match_host_pipelined(stt, h_text, n, h_out, cap, count, static_cast<cudaStream_t>(stream));
+    } catch (...) {
+        set_error("unexpected host exception");
+        return AC_ERR_NO_MEMORY;
     }
-    if (n && (e = cudaMemcpyAsync(d_text, h_text, n, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
-        cleanup();
-        return cuda_fail(e, "H2D text");
-    }
-    // a NULL h_out means count only; a non-NULL h_out with cap 0 still emits
-    ac_match_t *dst = h_out ? (d_out ? d_out : reinterpret_cast<ac_match_t *>(d_res + 1)) : nullptr;
-    rc = ac_match_async(stt, d_text, n, 0, 0, dst, cap, d_res, stream, nullptr);
-    if (rc == AC_OK) rc = finish_sync(d_res, count, s);
-    if (rc == AC_OK && h_out && count && *count) {
-        if ((e = cudaMemcpyAsync(h_out, d_out, *count * sizeof(ac_match_t), cudaMemcpyDeviceToHost, s)) != cudaSuccess) {
-            cleanup();
-            return cuda_fail(e, "D2H matches");
-        }
-    }
-    cleanup();
-    return rc;
 }
 
 }  // extern "C"

@@ -182,9 +182,11 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
         t.stt.assign((size_t)S * stride * eb, 0);
         t.out_off.assign(S + 1, 0);
         uint64_t n_out = 0;
+        t.max_out = 0;
         for (uint32_t i = 0; i < S; i++) {
             t.out_off[i] = (uint32_t)n_out;
             n_out += out[order[i]].size();
+            t.max_out = std::max<uint32_t>(t.max_out, (uint32_t)out[order[i]].size());
             if (n_out >= (1ull << 32)) {
                 set_error("output closure too large");
                 return AC_ERR_TOO_LARGE;

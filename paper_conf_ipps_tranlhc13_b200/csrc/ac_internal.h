@@ -15,6 +15,7 @@ struct ac_table {
     uint32_t n_classes = 0;
     uint32_t row_stride = 0;   // entries per row
     uint32_t info_col = 0;     // entry index of the output summary (payload u32, count)
+    uint32_t max_out = 0;      // max |output(s)|: bounds matches per byte (32-bit chain counters)
     uint32_t entry_bytes = 2;
     uint32_t forward = 0;
     uint8_t class_map[256] = {0};

@@ -232,9 +232,14 @@ __device__ __forceinline__ uint2 out_info_pred(const E *s_stt, const SttView &st
     return make_uint2(pay, c);
 }
 
-// One transition inside the owned chunk: count or emit output(s) at pos.
+// One transition inside the owned chunk: count or emit output(s) at the
+// byte whose record key is key0 = (global start) << 24.  cnt is the chain's
+// running count (32-bit: the planner keeps chain_len x max|output| < 2^31).
+// wp: MODE_EMIT -> the chain's next output index (counts down);
+//     MODE_EMIT_OPT -> the address of the LAST slot of the chain's scratch
+//     slot (record k goes to wp - 8k).
 template <typename E, int TIER, int MODE>
-__device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp, uint32_t byte, uint64_t pos,
+__device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp, uint32_t byte, uint64_t key0,
                                         bool live, const uint8_t *s_cmap, const E *s_stt, const SttView &st,
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
@@ -254,16 +259,15 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
         if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
             c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);
         if constexpr (MODE == MODE_EMIT_OPT) {
-            // wp = end of this chain's scratch slot; record k goes to wp-1-k
-            const uint64_t key0 = (so.base + pos) << 24;
+            uint64_t *last = reinterpret_cast<uint64_t *>(wp);
             const uint32_t one = (c == 1u) & (cnt < so.q ? 1u : 0u);
-            uint64_t *dst = so.scratch + (wp - 1 - cnt);
-            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}" ::"l"(dst),
+            asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.global.u64 [%0], %1;\n\t}" ::"l"(
+                             last - cnt),
                          "l"(key0 | o.x), "r"(one)
                          : "memory");
             if (c > 1u) {
                 for (uint32_t j = o.x + c; j > o.x; --j) {
-                    if (cnt < so.q) so.scratch[wp - 1 - cnt] = key0 | __ldg(st.out_ids + j - 1);
+                    if (cnt < so.q) last[-(int64_t)cnt] = key0 | __ldg(st.out_ids + j - 1);
                     cnt++;
                 }
             } else {
@@ -277,7 +281,6 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
     if ((e & EntryBits<E>::FLAG) && live) {
         const uint32_t c = out_count<E, TIER>(s_stt, st, s);
         if constexpr (MODE == MODE_EMIT) {
-            const uint64_t key0 = (so.base + pos) << 24;
             const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
             if (c == 1) {
                 so.out[--wp] = key0 | p;
@@ -285,15 +288,14 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint64_t &cnt, uint64_t &wp
                 for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
             }
         } else if constexpr (MODE == MODE_EMIT_OPT) {
-            // wp = end of this chain's scratch slot; record k goes to wp-1-k
-            const uint64_t key0 = (so.base + pos) << 24;
+            uint64_t *last = reinterpret_cast<uint64_t *>(wp);
             const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
             if (c == 1) {
-                if (cnt < so.q) so.scratch[wp - 1 - cnt] = key0 | p;
+                if (cnt < so.q) last[-(int64_t)cnt] = key0 | p;
                 cnt++;
             } else {
                 for (uint32_t j = p + c; j > p; --j) {
-                    if (cnt < so.q) so.scratch[wp - 1 - cnt] = key0 | __ldg(st.out_ids + j - 1);
+                    if (cnt < so.q) last[-(int64_t)cnt] = key0 | __ldg(st.out_ids + j - 1);
                     cnt++;
                 }
             }
@@ -317,11 +319,11 @@ __device__ __forceinline__ unsigned long long warp_sum(unsigned long long v) {
 // Walk text[a, b) right to left; OWNED selects emission (else warm-up).
 template <typename E, int TIER, int MODE, bool OWNED>
 __device__ __forceinline__ void walk_global(const uint8_t *__restrict__ text, uint64_t a, uint64_t b, uint32_t &s,
-                                            uint64_t &cnt, uint64_t &wp, const uint8_t *s_cmap, const E *s_stt,
+                                            uint32_t &cnt, uint64_t &wp, const uint8_t *s_cmap, const E *s_stt,
                                             const SttView &st, const ScanOut &so) {
     auto one = [&](uint32_t byte, uint64_t pos) {
         if constexpr (OWNED)
-            ac_step<E, TIER, MODE>(s, cnt, wp, byte, pos, true, s_cmap, s_stt, st, so);
+            ac_step<E, TIER, MODE>(s, cnt, wp, byte, (so.base + pos) << 24, true, s_cmap, s_stt, st, so);
         else
             s = ac_move<E, TIER>(s, byte, s_cmap, s_stt, st);
     };
@@ -359,7 +361,7 @@ __global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ 
     const uint64_t r_lo = in_a ? ra.lo : rb.lo, r_hi = in_a ? ra.hi : rb.hi;
     const uint64_t r_len = in_a ? ra.chain_len : rb.chain_len, r_n = in_a ? ra.n_chains : rb.n_chains;
     const uint64_t r_c0 = in_a ? ra.chain0 : rb.chain0;
-    uint64_t cnt = 0;
+    uint32_t cnt = 0;
     if (ci < r_n) {
         const uint64_t lo = r_lo + ci * r_len;
         const uint64_t own_hi = min(lo + r_len, r_hi);
@@ -367,14 +369,14 @@ __global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ 
         const uint64_t g = r_c0 + ci;
         uint64_t wp = 0;
         if constexpr (MODE == MODE_EMIT) wp = so.chain_end[g];
-        if constexpr (MODE == MODE_EMIT_OPT) wp = (g + 1) * so.q;
+        if constexpr (MODE == MODE_EMIT_OPT) wp = reinterpret_cast<uint64_t>(so.scratch + (g + 1) * so.q - 1);
         uint32_t s = 0;
         walk_global<E, TIER, MODE, false>(text, own_hi, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
         walk_global<E, TIER, MODE, true>(text, lo, own_hi, s, cnt, wp, s_cmap, s_stt, st, so);
         if constexpr (MODE == MODE_COUNT_CHAINS || MODE == MODE_EMIT_OPT) so.chain_counts[g] = cnt;
     }
     if constexpr (MODE == MODE_COUNT_TOTAL) {
-        const unsigned long long tot = warp_sum(cnt);
+        const unsigned long long tot = warp_sum((unsigned long long)cnt);
         if ((threadIdx.x & 31) == 0 && tot) atomicAdd(so.total, tot);
     }
 }
@@ -413,8 +415,8 @@ __global__ void __launch_bounds__(GT) k_rewalk(const uint8_t *__restrict__ text,
         const uint64_t sub = (own_hi - lo + GT - 1) / GT;
         const uint64_t a = min(lo + threadIdx.x * sub, own_hi), b = min(a + sub, own_hi);
         const uint64_t walk_hi = min(b + (uint64_t)st.halo, n_total);
-        uint64_t cnt = 0, wp = 0;
-        uint32_t s = 0;
+        uint64_t wp = 0;
+        uint32_t s = 0, cnt = 0;
         if (a < b) {
             walk_global<E, TIER, MODE_COUNT_CHAINS, false>(text, b, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
             walk_global<E, TIER, MODE_COUNT_CHAINS, true>(text, a, b, s, cnt, wp, s_cmap, s_stt, st, so);
@@ -468,24 +470,24 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
 }
 
 // ------------------------------------------- k_scan_staged (warp-private TMA)
-template <int WARPS, int K, int W, int NST>
+template <int WARPS, int K, int W, int NST, int SWIZZLE>
 struct StagedShape {
     static constexpr int ROWS = 32 * K;               // chains per warp = TMA box rows (<= 256)
     static constexpr int SLOT = ROWS * W;             // bytes per ring slot
     static constexpr int WARP_RING = NST * SLOT;
     static constexpr int RING = WARPS * WARP_RING;
     static constexpr int BARS = (WARPS * NST * 8 + 15) / 16 * 16;
-    static constexpr uint32_t SWZ = W == 128 ? 7u : W == 64 ? 3u : W == 32 ? 1u : 0u;
+    static constexpr uint32_t SWZ = !SWIZZLE ? 0u : W == 128 ? 7u : W == 64 ? 3u : W == 32 ? 1u : 0u;
     static_assert(ROWS <= 256, "TMA box rows");
     static_assert(W == 16 || W == 32 || W == 64 || W == 128, "tile width");
     static_assert(SLOT % 512 == 0 || W == 16, "slots must keep the swizzle atom aligned");
 };
 
-template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST>
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE>
 __global__ void __launch_bounds__(WARPS * 32, 1)
     k_scan_staged(const __grid_constant__ CUtensorMap tmap, const uint8_t *__restrict__ mtext, SttView st,
                   StagedGeom g, ScanOut so) {
-    using Sh = StagedShape<WARPS, K, W, NST>;
+    using Sh = StagedShape<WARPS, K, W, NST, SWIZZLE>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *ring = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     uint64_t *bars = reinterpret_cast<uint64_t *>(ring + Sh::RING);
@@ -531,8 +533,8 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     if (lane == 0)
         for (uint32_t j = 0; j < (uint32_t)NST && j < m; j++) issue(j);
 
-    uint32_t s[K], hlen[K];
-    uint64_t cnt[K], wp[K], cbase[K];
+    uint32_t s[K], hlen[K], cnt[K];
+    uint64_t wp[K], cbase[K];
     bool live[K];
 #pragma unroll
     for (int k = 0; k < K; k++) {
@@ -546,7 +548,8 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
         hlen[k] = (uint32_t)(rest < H ? rest : H);
         if constexpr (MODE == MODE_EMIT)
             if (live[k]) wp[k] = so.chain_end[g.chain0 + c];
-        if constexpr (MODE == MODE_EMIT_OPT) wp[k] = (g.chain0 + c + 1) * so.q;
+        if constexpr (MODE == MODE_EMIT_OPT)
+            wp[k] = reinterpret_cast<uint64_t>(so.scratch + (g.chain0 + c + 1) * so.q - 1);
         // the last chain's halo row is outside the tensor map (and any halo
         // wider than the next chain): warm up from global memory instead
         if (live[k] && (!tma_halo || c + 1 == g.n_chains)) {
@@ -583,19 +586,19 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
             for (int q = W / 16 - 1; q >= 0; --q) {
                 uint4 v[K];
+                uint64_t kb[K];  // record key of the chunk's first byte: (global start) << 24
 #pragma unroll
                 for (int k = 0; k < K; k++) {
                     const uint32_t logical = (k * 32 + lane) * W + q * 16;
                     v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
+                    kb[k] = (so.base + g.m0 + cbase[k] + col0 + q * 16) << 24;
                 }
 #pragma unroll
                 for (int bb = 15; bb >= 0; --bb) {
 #pragma unroll
-                    for (int k = 0; k < K; k++) {
-                        const uint64_t pos = g.m0 + cbase[k] + col0 + q * 16 + bb;
-                        ac_step<E, TIER, MODE>(s[k], cnt[k], wp[k], byte_of(v[k], bb), pos, live[k], s_cmap, s_stt,
-                                               st, so);
-                    }
+                    for (int k = 0; k < K; k++)
+                        ac_step<E, TIER, MODE>(s[k], cnt[k], wp[k], byte_of(v[k], bb), kb[k] + ((uint64_t)bb << 24),
+                                               live[k], s_cmap, s_stt, st, so);
                 }
             }
         }
@@ -691,11 +694,11 @@ cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_tota
     }
 }
 
-template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST>
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE>
 static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
                                    const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
-    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST>;
-    const StagedConfig cfg{WARPS, K, W, NST};
+    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE>;
+    const StagedConfig cfg{WARPS, K, W, NST, SWIZZLE};
     const size_t smem = staged_smem_bytes(cfg, smem_stt);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -710,8 +713,8 @@ template <typename E, int TIER, int MODE>
 static cudaError_t launch_staged_m(int variant, const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
                                    const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t s) {
     switch (variant) {
-#define AC_CASE(i, w, k, wd, ns) \
-    case i: return launch_staged_v<E, TIER, MODE, w, k, wd, ns>(tmap, mtext, st, g, so, smem_stt, s);
+#define AC_CASE(i, w, k, wd, ns, sw) \
+    case i: return launch_staged_v<E, TIER, MODE, w, k, wd, ns, sw>(tmap, mtext, st, g, so, smem_stt, s);
         AC_STAGED_VARIANTS(AC_CASE)
 #undef AC_CASE
     }

@@ -9,7 +9,7 @@
 namespace acx {
 
 static const StagedConfig kVariants[] = {
-#define AC_ROW(i, w, k, wd, ns) {w, k, wd, ns},
+#define AC_ROW(i, w, k, wd, ns, sw) {w, k, wd, ns, sw},
     AC_STAGED_VARIANTS(AC_ROW)
 #undef AC_ROW
 };

@@ -66,17 +66,19 @@ struct StagedConfig {
     int k;           // chains per lane
     int width;       // tile width W in bytes (16 / 32 / 64 = TMA swizzle span)
     int stages;      // ring slots per warp
+    int swizzle;     // 1 = TMA swizzle (conflict-free lane reads), 0 = plain rows (NEXT-1 ablation)
 };
 
-// AC_STAGED_VARIANTS(X): X(index, warps, chains per lane, tile width, ring depth)
+// AC_STAGED_VARIANTS(X): X(index, warps, chains per lane, tile width, ring depth, swizzle)
 #define AC_STAGED_VARIANTS(X) \
-    X(1, 16, 1, 32, 3)        \
-    X(2, 16, 2, 32, 2)        \
-    X(3, 32, 1, 32, 2)        \
-    X(4, 32, 1, 16, 3)        \
-    X(5, 16, 2, 16, 3)        \
-    X(6, 32, 2, 16, 2)        \
-    X(7, 32, 1, 16, 2)
+    X(1, 16, 1, 32, 3, 1)     \
+    X(2, 16, 2, 32, 2, 1)     \
+    X(3, 32, 1, 32, 2, 1)     \
+    X(4, 32, 1, 16, 3, 1)     \
+    X(5, 16, 2, 16, 3, 1)     \
+    X(6, 32, 2, 16, 2, 1)     \
+    X(7, 32, 1, 16, 2, 1)     \
+    X(8, 32, 1, 32, 2, 0)
 
 // Kernel entry points (host side launchers); all return cudaError_t.
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,

@@ -144,7 +144,7 @@ def test_c3_hybrid_and_global_tiers():
         assert_same(gpu_keys(stt, w.text), want)
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7])
+@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7, 8])
 @pytest.mark.parametrize("name,tier", [("c1", ac.TIER_AUTO), ("c2", ac.TIER_GLOBAL), ("c2s", ac.TIER_COMPACT)])
 def test_staged_variants(variant, name, tier):
     P = {"c1": None, "c2": 400, "c2s": 80}[name]
@@ -344,6 +344,22 @@ def test_host_entry_point():
     assert c == want.size
     assert_same(out[:c].numpy(), want)
     assert ac.match_host(stt, host, None) == want.size
+
+
+def test_host_entry_point_pipelined_chunks():
+    # > 32 MiB: several pipelined chunks (shards with halos) through ac_match_host
+    w = synth.make("c1", n=(70 << 20) + 5)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    want = oracle_keys(o, w.text)
+    host = torch.from_numpy(w.text).pin_memory()
+    out = torch.empty(want.size, dtype=torch.int64).pin_memory()
+    assert ac.match_host(stt, host, out) == want.size
+    assert_same(out.numpy(), want)
+    small = torch.empty(want.size // 2, dtype=torch.int64).pin_memory()
+    with pytest.raises(ac.CapacityError) as e:
+        ac.match_host(stt, host, small)
+    assert e.value.count == want.size
 
 
 def test_determinism():
