@@ -78,7 +78,8 @@ struct StagedConfig {
     X(5, 16, 2, 16, 3, 1)     \
     X(6, 32, 2, 16, 2, 1)     \
     X(7, 32, 1, 16, 2, 1)     \
-    X(8, 32, 1, 32, 2, 0)
+    X(8, 32, 1, 32, 2, 0)     \
+    X(9, 16, 2, 16, 2, 1)
 
 // Kernel entry points (host side launchers); all return cudaError_t.
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,
