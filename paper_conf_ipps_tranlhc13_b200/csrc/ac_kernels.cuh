@@ -80,8 +80,24 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
     } else if constexpr (TIER == AC_TIER_GLOBAL) {
         return __ldg(g_stt + idx);
     } else {
-        const E *p = (s < hot) ? (s_stt + idx) : (g_stt + idx);
-        return *p;
+        // HYBRID: two predicated loads, one per address space.  (A generic
+        // load would send the shared-memory lanes through the L1TEX tag
+        // stage too -- the stage that binds this tier, ncu: 97 % busy.)
+        const uint32_t in_smem = s < hot;
+        const uint32_t sa = smem_u32(s_stt + idx);
+        const uint64_t ga = reinterpret_cast<uint64_t>(g_stt + idx);
+        uint32_t v = 0;
+        if constexpr (sizeof(E) == 2)
+            asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%2];\n\t"
+                "@!p ld.global.nc.u16 %0, [%3];\n\t}"
+                : "+r"(v)
+                : "r"(in_smem), "r"(sa), "l"(ga));
+        else
+            asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\t@p ld.shared.u32 %0, [%2];\n\t"
+                "@!p ld.global.nc.u32 %0, [%3];\n\t}"
+                : "+r"(v)
+                : "r"(in_smem), "r"(sa), "l"(ga));
+        return v;
     }
 }
 
