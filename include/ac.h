@@ -93,6 +93,11 @@ typedef struct {
                               come out in canonical (start, pattern) order;
                               1 = the paper's forward automaton (tests only:
                               ac_build rejects it, ac_compile accepts it)    */
+    uint32_t stride;       /* bytes per dependent lookup in the staged scan:
+                              0 = auto (2 for GLOBAL-tier automata with
+                              <= 8 classes whose two-byte table fits 64 MiB),
+                              1, or 2 (needs 32-bit
+                              entries -- set entry_bytes = 4 for small S)    */
 } ac_build_opts;
 
 typedef struct {
@@ -122,6 +127,9 @@ typedef struct {
     uint32_t compact_dense, compact_od, compact_os, compact_dstride;
     uint32_t compact_sparse_off, compact_out_off;
     uint64_t compact_bytes;
+    uint32_t stride;       /* 1 or 2 (two-byte table present)                */
+    uint32_t stride2_cols; /* row stride of the two-byte table (C*C, odd)   */
+    uint64_t stt2_bytes;
 } ac_stt_info;
 
 /* Scan variants (SURVEY 8(f) NEXT-1 ablations are selectable here). */
@@ -148,6 +156,8 @@ typedef struct {
                               re-scanned straight into place                 */
     uint32_t two_pass;     /* list mode: 1 = count pass + emit pass instead
                               of the single pass (ablation / fallback)       */
+    uint32_t stride;       /* 0 = the table's default, 1 = force one byte
+                              per lookup even if a two-byte table exists     */
     uint32_t n_events;     /* pairs available in `events`                    */
     void **events;         /* optional cudaEvent_t[2 * n_events]: events[2i]
                               and events[2i+1] are recorded on the stream
@@ -237,6 +247,10 @@ ac_status ac_table_query(const ac_table *t, ac_stt_info *info);
 ac_status ac_table_export(const ac_table *t, uint8_t *class_map, void *stt, uint32_t *out_off,
                           uint32_t *out_ids);
 ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm);
+/* opts->stride == 2 also builds the two-byte table (NEXT-4): n_states rows of
+ * stride2_cols u32, column c1*C + c2 -> delta(delta(s,c1),c2) | bit 31 =
+ * output(final) != {} | bit 30 = output(middle) != {}. */
+ac_status ac_table_export_stride2(const ac_table *t, uint32_t *tab);
 void ac_table_free(ac_table *t);
 
 /* ------------------------------------------------------------ diagnostics */

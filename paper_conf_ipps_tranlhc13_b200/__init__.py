@@ -34,7 +34,7 @@ TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global", 4: "compact"}
 EXPORTED = [
     "ac_build", "ac_free", "ac_stt_query", "ac_stt_pattern_lengths", "ac_match", "ac_match_shard",
     "ac_match_async", "ac_last_launch_count", "ac_last_launch_name", "ac_match_host", "ac_compile", "ac_table_query",
-    "ac_table_export", "ac_table_export_compact", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
+    "ac_table_export", "ac_table_export_compact", "ac_table_export_stride2", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
 ]
 
 
@@ -52,7 +52,7 @@ class CapacityError(AcError):
 
 class ac_build_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("entry_bytes", ctypes.c_uint32), ("tier", ctypes.c_uint32),
-                ("hot_rows", ctypes.c_uint32), ("forward", ctypes.c_uint32)]
+                ("hot_rows", ctypes.c_uint32), ("forward", ctypes.c_uint32), ("stride", ctypes.c_uint32)]
 
 
 class ac_stt_info(ctypes.Structure):
@@ -62,12 +62,14 @@ class ac_stt_info(ctypes.Structure):
                 ("info_col", ctypes.c_uint32), ("stt_bytes", ctypes.c_uint64), ("out_entries", ctypes.c_uint64),
                 ("compact_dense", ctypes.c_uint32), ("compact_od", ctypes.c_uint32), ("compact_os", ctypes.c_uint32),
                 ("compact_dstride", ctypes.c_uint32), ("compact_sparse_off", ctypes.c_uint32),
-                ("compact_out_off", ctypes.c_uint32), ("compact_bytes", ctypes.c_uint64)]
+                ("compact_out_off", ctypes.c_uint32), ("compact_bytes", ctypes.c_uint64),
+                ("stride", ctypes.c_uint32), ("stride2_cols", ctypes.c_uint32), ("stt2_bytes", ctypes.c_uint64)]
 
 
 class ac_match_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("kernel", ctypes.c_uint32), ("chain_bytes", ctypes.c_uint32),
                 ("variant", ctypes.c_uint32), ("scratch_slots", ctypes.c_uint32), ("two_pass", ctypes.c_uint32),
+                ("stride", ctypes.c_uint32),
                 ("n_events", ctypes.c_uint32),
                 ("events", ctypes.POINTER(ctypes.c_void_p))]
 
@@ -94,6 +96,7 @@ def lib():
         L.ac_table_query.argtypes = [_vp, ctypes.POINTER(ac_stt_info)]
         L.ac_table_export.argtypes = [_vp, _vp, _vp, _vp, _vp]
         L.ac_table_export_compact.argtypes = [_vp, _vp, _vp]
+        L.ac_table_export_stride2.argtypes = [_vp, _vp]
         L.ac_stt_pattern_lengths.argtypes = [_vp, _vp]
         L.ac_match.argtypes = [_vp, _vp, _u64, _vp, _u64, _u64p, _vp]
         L.ac_match_shard.argtypes = [_vp, _vp, _u64, _u64, _u64, _vp, _u64, _u64p, _vp]
@@ -137,8 +140,8 @@ def _pattern_arrays(patterns):
     return pats, bufs, ptrs, lens
 
 
-def _opts(entry_bytes=0, tier=TIER_AUTO, hot_rows=0, forward=False):
-    return ac_build_opts(ctypes.sizeof(ac_build_opts), entry_bytes, tier, hot_rows, 1 if forward else 0)
+def _opts(entry_bytes=0, tier=TIER_AUTO, hot_rows=0, forward=False, stride=0):
+    return ac_build_opts(ctypes.sizeof(ac_build_opts), entry_bytes, tier, hot_rows, 1 if forward else 0, stride)
 
 
 def _info_dict(info: ac_stt_info) -> dict:
@@ -148,11 +151,12 @@ def _info_dict(info: ac_stt_info) -> dict:
 class Stt:
     """A device STT (phase-1 result), immutable, freed with the object."""
 
-    def __init__(self, patterns, device: int = 0, entry_bytes: int = 0, tier: int = TIER_AUTO, hot_rows: int = 0):
+    def __init__(self, patterns, device: int = 0, entry_bytes: int = 0, tier: int = TIER_AUTO, hot_rows: int = 0,
+                 stride: int = 0):
         L = lib()
         self.patterns, bufs, ptrs, lens = _pattern_arrays(patterns)
         h = ctypes.c_void_p()
-        o = _opts(entry_bytes, tier, hot_rows)
+        o = _opts(entry_bytes, tier, hot_rows, stride=stride)
         _check(L.ac_build(ptrs, lens, len(self.patterns), int(device), ctypes.byref(o), ctypes.byref(h)))
         self._h = h
         self.device = int(device)
@@ -195,9 +199,9 @@ def _check_text(text: torch.Tensor):
 
 
 def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, scratch_slots: int = 0,
-           two_pass: bool = False, events=None):
+           two_pass: bool = False, events=None, stride: int = 0):
     o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, scratch_slots,
-                      1 if two_pass else 0, 0, None)
+                      1 if two_pass else 0, stride, 0, None)
     if events:
         arr = (ctypes.c_void_p * (2 * len(events)))(*[e.cuda_event for pair in events for e in pair])
         o.n_events = len(events)
@@ -208,7 +212,8 @@ def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, sc
 
 def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: torch.Tensor, *,
                 n_halo: int = 0, base: int = 0, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0,
-                variant: int = 0, scratch_slots: int = 0, two_pass: bool = False, events=None) -> int:
+                variant: int = 0, scratch_slots: int = 0, two_pass: bool = False, stride: int = 0,
+                events=None) -> int:
     """Enqueue the scan; result (int64[2] CUDA) receives (count, status).
     ``text`` holds n_owned + n_halo bytes.  ``kernel``/``chain_bytes``/
     ``variant``/``scratch_slots``/``two_pass`` select the scan (ac_match_opts).  ``events``: optional list
@@ -229,7 +234,7 @@ def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: 
         cap = out.numel()
         # non-NULL selects list mode; with cap == 0 the status gates every write
         optr = out.data_ptr() if cap else result.data_ptr()
-    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events)
+    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events, stride)
     L = lib()
     _check(L.ac_match_async(stt.handle, text.data_ptr() if n_total else None, n_total - n_halo, n_halo, base,
                             optr, cap, result.data_ptr(), _stream_ptr(stream), ctypes.byref(o)))
@@ -313,16 +318,18 @@ class HostTable:
     out_off: "object"
     out_ids: "object"
     compact: "object" = None   # COMPACT blob (uint8) if requested
+    stt2: "object" = None      # two-byte table (uint32, S x stride2_cols) if requested
     perm: "object" = None      # compact id -> dense BFS id
 
 
-def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact: bool = False) -> HostTable:
+def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact: bool = False,
+                  stride: int = 0) -> HostTable:
     """Phase 1 on the host only (no device) -- for builder tests."""
     import numpy as np
     L = lib()
     pats, bufs, ptrs, lens = _pattern_arrays(patterns)
     h = ctypes.c_void_p()
-    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=TIER_COMPACT if compact else TIER_AUTO)
+    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=TIER_COMPACT if compact else TIER_AUTO, stride=stride)
     _check(L.ac_compile(ptrs, lens, len(pats), ctypes.byref(o), ctypes.byref(h)))
     try:
         info = ac_stt_info()
@@ -339,6 +346,12 @@ def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact
             blob = np.zeros(d["compact_bytes"], dtype=np.uint8)
             perm = np.zeros(d["n_states"], dtype=np.uint32)
             _check(L.ac_table_export_compact(h, blob.ctypes.data, perm.ctypes.data))
-        return HostTable(d, cm, stt.reshape(d["n_states"], d["row_stride"]), off, ids[:d["out_entries"]], blob, perm)
+        t2 = None
+        if d["stride"] == 2:
+            t2 = np.zeros(d["n_states"] * d["stride2_cols"], dtype=np.uint32)
+            _check(L.ac_table_export_stride2(h, t2.ctypes.data))
+            t2 = t2.reshape(d["n_states"], d["stride2_cols"])
+        return HostTable(d, cm, stt.reshape(d["n_states"], d["row_stride"]), off, ids[:d["out_entries"]],
+                         compact=blob, stt2=t2, perm=perm)
     finally:
         L.ac_table_free(h)

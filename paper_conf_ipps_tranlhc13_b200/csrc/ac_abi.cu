@@ -144,6 +144,9 @@ static SttView view_of(const ac_stt *h, int v) {
     s.c_dstride = h->host.c_dstride;
     s.c_sparse_off = h->host.c_sparse_off;
     s.c_out_off = h->host.c_out_off;
+    s.stt2 = v ? h->d_stt2 : nullptr;  // only the staged kernel walks two bytes per lookup
+    s.stride2 = h->host.stride2;
+    s.n_classes = h->host.n_classes;
     if (h->tier == AC_TIER_COMPACT) {
         s.smem_rows = h->host.n_states;
         s.smem_bytes = (uint32_t)h->host.compact.size();
@@ -168,6 +171,8 @@ static uint32_t tier_of(const ac_stt *h, const SttView &v) {
 
 static void free_device(ac_stt *h) {
     cudaFree(h->d_stt);
+    cudaFree(h->d_stt2);
+    h->d_stt2 = nullptr;
     cudaFree(h->d_class_map);
     cudaFree(h->d_out_off);
     cudaFree(h->d_out_ids);
@@ -232,7 +237,9 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         set_error("staged variant " + std::to_string(variant) + " has no room for the COMPACT table");
         return AC_ERR_INVALID_ARG;
     }
-    const SttView sg = view_of(h, 0), ss = view_of(h, variant);
+    SttView sg = view_of(h, 0), ss = view_of(h, variant);
+    // the two-byte walk exists for the two 32-warp x 16-byte shapes only
+    if ((opts && opts->stride == 1) || (variant != 4 && variant != 7)) ss.stt2 = nullptr;
     const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
     const size_t smem_g = smem_of(h, sg), smem_s = smem_of(h, ss);
     const StagedConfig cfg = staged_variant(variant);
@@ -599,6 +606,10 @@ ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint3
             set_error("the automaton does not fit the COMPACT shared-memory encoding");
             rc = AC_ERR_TOO_LARGE;
         }
+        if (rc == AC_OK && opts && opts->stride == 2 && !stride2_table(*t, 64ull << 20)) {
+            set_error("stride 2 needs 32-bit entries and a two-byte table <= 64 MiB");
+            rc = AC_ERR_INVALID_ARG;
+        }
     } catch (...) {
         set_error("host allocation failed");
         rc = AC_ERR_NO_MEMORY;
@@ -630,6 +641,15 @@ static void fill_info(const ac_table &t, ac_stt_info *info) {
     info->compact_sparse_off = t.c_sparse_off;
     info->compact_out_off = t.c_out_off;
     info->compact_bytes = t.compact.size();
+    info->stride = t.stride2 ? 2 : 1;
+    info->stride2_cols = t.stride2;
+    info->stt2_bytes = (uint64_t)t.stt2.size() * 4;
+}
+
+ac_status ac_table_export_stride2(const ac_table *t, uint32_t *tab) {
+    if (!t || t->stt2.empty() || !tab) return AC_ERR_INVALID_ARG;
+    std::memcpy(tab, t->stt2.data(), t->stt2.size() * 4);
+    return AC_OK;
 }
 
 ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm) {
@@ -737,6 +757,21 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     }
     h->tier = tier;
     h->hot_rows = hot;
+    // NEXT-4: two bytes per lookup for small alphabets on the L1/L2 tier
+    const uint32_t want_stride = opts ? opts->stride : 0;
+    if (want_stride > 2) {
+        delete h;
+        set_error("stride must be 0, 1 or 2");
+        return AC_ERR_INVALID_ARG;
+    }
+    if (want_stride == 2 || (want_stride == 0 && tier == AC_TIER_GLOBAL && t.n_classes <= 8)) {
+        const bool ok = tier == AC_TIER_GLOBAL && stride2_table(h->host, 64ull << 20);
+        if (!ok && want_stride == 2) {
+            delete h;
+            set_error("stride 2 needs the GLOBAL tier, 32-bit entries and a two-byte table <= 64 MiB");
+            return AC_ERR_INVALID_ARG;
+        }
+    }
 
     int prev = -1;
     cudaGetDevice(&prev);
@@ -754,6 +789,11 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     if ((e = cudaMemset(h->d_stt, 0, stt_alloc)) != cudaSuccess) return fail(e, "cudaMemset(stt)");
     if ((e = cudaMemcpy(h->d_stt, blob.data(), blob.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
         return fail(e, "H2D stt");
+    if (!t.stt2.empty()) {
+        if ((e = cudaMalloc(&h->d_stt2, t.stt2.size() * 4)) != cudaSuccess) return fail(e, "cudaMalloc(stt2)");
+        if ((e = cudaMemcpy(h->d_stt2, t.stt2.data(), t.stt2.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
+            return fail(e, "H2D stt2");
+    }
     if ((e = cudaMalloc(&h->d_class_map, 256)) != cudaSuccess) return fail(e, "cudaMalloc(class map)");
     if ((e = cudaMemcpy(h->d_class_map, t.class_map, 256, cudaMemcpyHostToDevice)) != cudaSuccess)
         return fail(e, "H2D class map");

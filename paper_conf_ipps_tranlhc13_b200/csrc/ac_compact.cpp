@@ -157,4 +157,38 @@ bool compact_table(ac_table &t, size_t budget) {
     return true;
 }
 
+// NEXT-4: the two-byte next-move table, T2(s, c1 c2) =
+// delta(delta(s, c1), c2), so a small-alphabet scan does one dependent gather
+// per TWO bytes (the paper's O(n) walk, with half the steps).  Bit 31
+// flags output(final) != {}, bit 30 flags output(middle) != {} (the kernel
+// recovers the middle state from the one-byte table in that rare case).
+// Built from the dense one-byte table; requires 32-bit entries.
+bool stride2_table(ac_table &t, size_t max_bytes) {
+    const uint32_t S = t.n_states, C = t.n_classes, stride = t.row_stride;
+    if (t.entry_bytes != 4 || S == 0 || S >= (1u << 30)) return false;
+    const uint64_t cols = (uint64_t)C * C;
+    const uint32_t stride2 = (uint32_t)(cols | 1u);
+    if ((uint64_t)S * stride2 * 4 > max_bytes || (uint64_t)S * stride2 >= (1ull << 32)) return false;
+    auto delta = [&](uint32_t s, uint32_t c) -> uint32_t {
+        uint32_t e;
+        std::memcpy(&e, &t.stt[((size_t)s * stride + c) * 4], 4);
+        return e;
+    };
+    std::vector<uint32_t> tab((size_t)S * stride2, 0);
+    for (uint32_t s = 0; s < S; s++) {
+        uint32_t *row = &tab[(size_t)s * stride2];
+        for (uint32_t c1 = 0; c1 < C; c1++) {
+            const uint32_t e1 = delta(s, c1);
+            const uint32_t mid = e1 & 0x7fffffffu;
+            for (uint32_t c2 = 0; c2 < C; c2++) {
+                const uint32_t e2 = delta(mid, c2);
+                row[c1 * C + c2] = (e2 & 0x7fffffffu) | ((e2 >> 31) << 31) | ((e1 >> 31) << 30);
+            }
+        }
+    }
+    t.stt2.swap(tab);
+    t.stride2 = stride2;
+    return true;
+}
+
 }  // namespace acx

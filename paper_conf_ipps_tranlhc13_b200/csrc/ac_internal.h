@@ -35,6 +35,12 @@ struct ac_table {
     uint32_t c_sparse_off = 0, c_out_off = 0;  // byte offsets inside `compact`
     std::vector<uint8_t> compact;
     std::vector<uint32_t> c_perm;              // compact id -> BFS id
+
+    // two-byte table (NEXT-4), built by stride2_table(): row s, column
+    // c1 * n_classes + c2 -> delta(delta(s,c1),c2) | final flag << 31 |
+    // middle flag << 30; rows padded to an odd number of words
+    uint32_t stride2 = 0;
+    std::vector<uint32_t> stt2;
 };
 
 // Device-side STT (library owned).
@@ -44,6 +50,7 @@ struct ac_stt {
     uint32_t tier = AC_TIER_GLOBAL;
     uint32_t hot_rows = 0;
     void *d_stt = nullptr;           // entries
+    uint32_t *d_stt2 = nullptr;      // two-byte table (NEXT-4) or NULL
     uint8_t *d_class_map = nullptr;  // 256 B
     uint32_t *d_out_off = nullptr;
     uint32_t *d_out_ids = nullptr;
@@ -57,4 +64,5 @@ void set_error(const std::string &msg);
 ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n,
                         const ac_build_opts *opts, ac_table &t);
 bool compact_table(ac_table &t, size_t budget);
+bool stride2_table(ac_table &t, size_t max_bytes);
 }  // namespace acx

@@ -248,6 +248,35 @@ __device__ __forceinline__ uint2 out_info_pred(const E *s_stt, const SttView &st
     return make_uint2(pay, c);
 }
 
+// Count or emit every pattern of output(x) at key0 (the branchy path).
+template <typename E, int TIER, int MODE>
+__device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t &cnt, uint64_t &wp, const E *s_stt,
+                                             const SttView &st, const ScanOut &so) {
+    const uint32_t c = out_count<E, TIER>(s_stt, st, x);
+    if constexpr (MODE == MODE_EMIT) {
+        const uint32_t p = out_payload<E, TIER>(s_stt, st, x);
+        if (c == 1) {
+            so.out[--wp] = key0 | p;
+        } else {
+            for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
+        }
+    } else if constexpr (MODE == MODE_EMIT_OPT) {
+        uint64_t *last = reinterpret_cast<uint64_t *>(wp);
+        const uint32_t p = out_payload<E, TIER>(s_stt, st, x);
+        if (c == 1) {
+            if (cnt < so.q) last[-(int64_t)cnt] = key0 | p;
+            cnt++;
+        } else {
+            for (uint32_t j = p + c; j > p; --j) {
+                if (cnt < so.q) last[-(int64_t)cnt] = key0 | __ldg(st.out_ids + j - 1);
+                cnt++;
+            }
+        }
+    } else {
+        cnt += c;
+    }
+}
+
 // One transition inside the owned chunk: count or emit output(s) at the
 // byte whose record key is key0 = (global start) << 24.  cnt is the chain's
 // running count (32-bit: the planner keeps chain_len x max|output| < 2^31).
@@ -294,31 +323,30 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
         }
         return;
     }
-    if ((e & EntryBits<E>::FLAG) && live) {
-        const uint32_t c = out_count<E, TIER>(s_stt, st, s);
-        if constexpr (MODE == MODE_EMIT) {
-            const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
-            if (c == 1) {
-                so.out[--wp] = key0 | p;
-            } else {
-                for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
-            }
-        } else if constexpr (MODE == MODE_EMIT_OPT) {
-            uint64_t *last = reinterpret_cast<uint64_t *>(wp);
-            const uint32_t p = out_payload<E, TIER>(s_stt, st, s);
-            if (c == 1) {
-                if (cnt < so.q) last[-(int64_t)cnt] = key0 | p;
-                cnt++;
-            } else {
-                for (uint32_t j = p + c; j > p; --j) {
-                    if (cnt < so.q) last[-(int64_t)cnt] = key0 | __ldg(st.out_ids + j - 1);
-                    cnt++;
-                }
-            }
-        } else {
-            cnt += c;
+    if ((e & EntryBits<E>::FLAG) && live) emit_outputs<E, TIER, MODE>(s, key0, cnt, wp, s_stt, st, so);
+}
+
+// NEXT-4: one lookup for two bytes.  T2[s][c1*C + c2] =
+// delta(delta(s,c1),c2) with bit 31 = output(final) != {} and bit 30 =
+// output(middle) != {}; the (rare) middle state is recovered from the
+// one-byte table.  b1 is the byte at key1's position, b2 the next one to the
+// left (the walk is right to left).
+static constexpr uint32_t T2_FIN = 1u << 31, T2_MID = 1u << 30, T2_MASK = (1u << 30) - 1;
+
+template <typename E, int TIER, int MODE>
+__device__ __forceinline__ void ac_step2(uint32_t &s, uint32_t &cnt, uint64_t &wp, uint32_t b1, uint32_t b2,
+                                         uint64_t key1, uint64_t key2, bool live, const uint8_t *s_cmap,
+                                         const E *s_stt, const SttView &st, const ScanOut &so) {
+    const uint32_t c1 = s_cmap[b1], c2 = s_cmap[b2];
+    const uint32_t e = __ldg(st.stt2 + s * st.stride2 + c1 * st.n_classes + c2);
+    if ((e & (T2_FIN | T2_MID)) && live) {
+        if (e & T2_MID) {
+            const uint32_t mid = next_entry<E, TIER>(s_stt, st, s, c1) & EntryBits<E>::MASK;
+            emit_outputs<E, TIER, MODE>(mid, key1, cnt, wp, s_stt, st, so);
         }
+        if (e & T2_FIN) emit_outputs<E, TIER, MODE>(e & T2_MASK, key2, cnt, wp, s_stt, st, so);
     }
+    s = e & T2_MASK;
 }
 
 __device__ __forceinline__ uint32_t byte_of(const uint4 &v, int bb) {
@@ -499,7 +527,7 @@ struct StagedShape {
     static_assert(SLOT % 512 == 0 || W == 16, "slots must keep the swizzle atom aligned");
 };
 
-template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE>
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1>
 __global__ void __launch_bounds__(WARPS * 32, 1)
     k_scan_staged(const __grid_constant__ CUtensorMap tmap, const uint8_t *__restrict__ mtext, SttView st,
                   StagedGeom g, ScanOut so) {
@@ -609,12 +637,23 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                     v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
                     kb[k] = (so.base + g.m0 + cbase[k] + col0 + q * 16) << 24;
                 }
+                if constexpr (STRIDE == 2) {
 #pragma unroll
-                for (int bb = 15; bb >= 0; --bb) {
+                    for (int bb = 15; bb >= 1; bb -= 2) {
 #pragma unroll
-                    for (int k = 0; k < K; k++)
-                        ac_step<E, TIER, MODE>(s[k], cnt[k], wp[k], byte_of(v[k], bb), kb[k] + ((uint64_t)bb << 24),
-                                               live[k], s_cmap, s_stt, st, so);
+                        for (int k = 0; k < K; k++)
+                            ac_step2<E, TIER, MODE>(s[k], cnt[k], wp[k], byte_of(v[k], bb), byte_of(v[k], bb - 1),
+                                                    kb[k] + ((uint64_t)bb << 24), kb[k] + ((uint64_t)(bb - 1) << 24),
+                                                    live[k], s_cmap, s_stt, st, so);
+                    }
+                } else {
+#pragma unroll
+                    for (int bb = 15; bb >= 0; --bb) {
+#pragma unroll
+                        for (int k = 0; k < K; k++)
+                            ac_step<E, TIER, MODE>(s[k], cnt[k], wp[k], byte_of(v[k], bb),
+                                                   kb[k] + ((uint64_t)bb << 24), live[k], s_cmap, s_stt, st, so);
+                    }
                 }
             }
         }
@@ -710,10 +749,10 @@ cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_tota
     }
 }
 
-template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE>
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1>
 static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
                                    const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
-    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE>;
+    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE, STRIDE>;
     const StagedConfig cfg{WARPS, K, W, NST, SWIZZLE};
     const size_t smem = staged_smem_bytes(cfg, smem_stt);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -728,6 +767,15 @@ static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext
 template <typename E, int TIER, int MODE>
 static cudaError_t launch_staged_m(int variant, const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
                                    const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t s) {
+    if (st.stt2) {
+        // the two-byte walk is instantiated for the L1/L2 tier with 32-bit
+        // entries (large small-alphabet automata, e.g. DNA) and two shapes
+        if constexpr (TIER == AC_TIER_GLOBAL && sizeof(E) == 4) {
+            if (variant == 4) return launch_staged_v<E, TIER, MODE, 32, 1, 16, 3, 1, 2>(tmap, mtext, st, g, so, smem_stt, s);
+            if (variant == 7) return launch_staged_v<E, TIER, MODE, 32, 1, 16, 2, 1, 2>(tmap, mtext, st, g, so, smem_stt, s);
+        }
+        return cudaErrorInvalidValue;
+    }
     switch (variant) {
 #define AC_CASE(i, w, k, wd, ns, sw) \
     case i: return launch_staged_v<E, TIER, MODE, w, k, wd, ns, sw>(tmap, mtext, st, g, so, smem_stt, s);

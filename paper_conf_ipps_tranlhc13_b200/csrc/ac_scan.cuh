@@ -30,6 +30,9 @@ struct SttView {
     uint32_t smem_bytes;      // STT bytes staged into shared memory
     // COMPACT tier (ac_compact.cpp): dense/sparse split and blob offsets
     uint32_t c_dense, c_od, c_dstride, c_sparse_off, c_out_off;
+    // two-byte table (NEXT-4): row s, column c1 * n_classes + c2; NULL = off
+    const uint32_t *stt2;
+    uint32_t stride2, n_classes;
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.

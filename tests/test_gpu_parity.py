@@ -135,6 +135,34 @@ def test_compact_edge_cases():
         assert_same(gpu_keys(stt, text, kernel=k), oracle_keys(o, text))
 
 
+@pytest.mark.parametrize("variant", [0, 4, 7, 3])
+def test_stride2_dna(variant):
+    """NEXT-4: two bytes per lookup -- matches at odd and even offsets,
+    middle and final positions, chains and halos of both parities."""
+    pats = [b"A", b"AC", b"CAG", b"GTTA", b"T" * 9, b"ACGTACGTAC", b"NN", b"GATTACA"]
+    o = Oracle(pats)
+    stt = ac.build(pats, tier=ac.TIER_GLOBAL, entry_bytes=4, stride=2)
+    assert stt.info["stride"] == 2
+    rng = np.random.default_rng(21)
+    text = np.frombuffer(b"ACGT", np.uint8)[rng.integers(0, 4, size=(1 << 20) + 7)].copy()
+    text[1000:1010] = ord("T")
+    text[77777:77784] = np.frombuffer(b"GATTACA", np.uint8)
+    text[5:7] = ord("N")
+    want = oracle_keys(o, text)
+    got = gpu_keys(stt, text, kernel=ac.KERNEL_STAGED, variant=variant)
+    assert_same(got, want)
+    assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED, variant=variant, chain_bytes=80), want)
+    assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED, stride=1), want)
+
+
+def test_stride2_is_auto_for_c4():
+    w = synth.make("c4", n=(2 << 20) + 3)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    assert stt.tier_name == "global" and stt.info["stride"] == 2
+    assert_same(gpu_keys(stt, w.text), oracle_keys(o, w.text))
+
+
 def test_c3_hybrid_and_global_tiers():
     w = synth.make("c3", n=(1 << 20) + 5)
     o = Oracle(w.patterns)

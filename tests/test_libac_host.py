@@ -199,6 +199,29 @@ def test_compact_encoding_equals_dense(which):
         assert S > 15000 and d["stt_bytes"] > 1_000_000  # the dense table would not fit
 
 
+@pytest.mark.parametrize("which", ["dna", "tiny"])
+def test_stride2_table_is_delta_composed(which):
+    """NEXT-4 table: T2(s, c1 c2) = delta(delta(s,c1),c2) with both flags."""
+    import synth
+    if which == "dna":
+        w = synth.make("c4", n=1 << 16, n_patterns=300)
+        pats = w.patterns
+    else:
+        pats = [b"AC", b"CA", b"A", b"GTT", b"TTTT"]
+    t = ac.compile_table(pats, entry_bytes=4, stride=2)
+    d = t.info
+    C, S = d["n_classes"], d["n_states"]
+    assert d["stride"] == 2 and d["stride2_cols"] >= C * C and d["stride2_cols"] % 2 == 1
+    T1 = t.stt[:, :C].astype(np.int64)
+    nxt, flag = T1 & 0x7FFFFFFF, (T1 >> 31) & 1
+    T2 = t.stt2[:, :C * C].astype(np.int64).reshape(S, C, C)
+    mid = nxt  # [s, c1]
+    want_state = nxt[mid]  # [s, c1, c2]
+    assert np.array_equal(T2 & ((1 << 30) - 1), want_state)
+    assert np.array_equal((T2 >> 31) & 1, flag[mid])
+    assert np.array_equal((T2 >> 30) & 1, np.broadcast_to(flag[:, :, None], (S, C, C)))
+
+
 def test_classes_and_stride():
     t = ac.compile_table([b"abc", b"zz"])
     assert t.info["n_classes"] == 5  # a, b, c, z + class 0
