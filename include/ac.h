@@ -216,6 +216,18 @@ ac_status ac_match_async(const ac_stt *stt, const uint8_t *d_text, uint64_t n_ow
                          uint64_t n_halo, uint64_t base, ac_match_t *d_out, uint64_t cap,
                          ac_result *d_result, void *stream, const ac_match_opts *opts);
 
+/* ac_match_segments: a batch of independent texts -- e.g. network packets,
+ * the NIDS workload of P:108 -- concatenated in d_text.
+ * d_seg_off (DEVICE, n_seg + 1 ascending uint64, first 0) gives the
+ * boundaries; segment i = d_text[d_seg_off[i], d_seg_off[i+1]) is scanned
+ * from the start state on its own, so no occurrence crosses a boundary.
+ * Records carry start offsets into d_text; the list is canonical.  Each
+ * segment must be shorter than 2^31 / max|output(s)| bytes.  Asynchronous
+ * like ac_match_async (count/status in *d_result); d_out == NULL = count
+ * only. */
+ac_status ac_match_segments(const ac_stt *stt, const uint8_t *d_text, const uint64_t *d_seg_off, uint64_t n_seg,
+                            ac_match_t *d_out, uint64_t cap, ac_result *d_result, void *stream);
+
 /* Number of kernel launches the last ac_match_async on this thread issued,
  * and the name of launch i (NULL if out of range). */
 uint32_t ac_last_launch_count(void);

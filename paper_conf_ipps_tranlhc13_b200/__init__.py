@@ -33,7 +33,7 @@ TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global", 4: "compact"}
 
 EXPORTED = [
     "ac_build", "ac_free", "ac_stt_query", "ac_stt_pattern_lengths", "ac_match", "ac_match_shard",
-    "ac_match_async", "ac_last_launch_count", "ac_last_launch_name", "ac_match_host", "ac_compile", "ac_table_query",
+    "ac_match_async", "ac_match_segments", "ac_last_launch_count", "ac_last_launch_name", "ac_match_host", "ac_compile", "ac_table_query",
     "ac_table_export", "ac_table_export_compact", "ac_table_export_stride2", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
 ]
 
@@ -102,6 +102,7 @@ def lib():
         L.ac_match_shard.argtypes = [_vp, _vp, _u64, _u64, _u64, _vp, _u64, _u64p, _vp]
         L.ac_match_async.argtypes = [_vp, _vp, _u64, _u64, _u64, _vp, _u64, _vp, _vp, ctypes.POINTER(ac_match_opts)]
         L.ac_match_host.argtypes = [_vp, _vp, _u64, _vp, _u64, _u64p, _vp]
+        L.ac_match_segments.argtypes = [_vp, _vp, _vp, _u64, _vp, _u64, _vp, _vp]
         L.ac_last_launch_count.restype = _u32
         L.ac_last_launch_count.argtypes = []
         L.ac_last_launch_name.restype = ctypes.c_char_p
@@ -259,6 +260,32 @@ def match(stt: Stt, text: torch.Tensor, out: torch.Tensor | None = None, *, n_ha
         out = torch.empty(max(1, need), dtype=torch.int64, device=text.device)
         res.zero_()
     match_async(stt, text, out, res, n_halo=n_halo, base=base, stream=stream, **knobs)
+    c, st = (int(x) for x in res.tolist())
+    if st == AC_ERR_CAPACITY:
+        raise CapacityError(st, f"{c} records do not fit in {out.numel()}", c)
+    _check(st)
+    return c, out[:c]
+
+
+def match_segments(stt: Stt, text: torch.Tensor, seg_off: torch.Tensor, out: torch.Tensor | None = None, *,
+                   stream=None):
+    """Packet batch (NEXT-2): segment i = text[seg_off[i]:seg_off[i+1]] is
+    scanned on its own (no match crosses a boundary).  seg_off: int64 CUDA
+    tensor of n_seg + 1 ascending offsets.  Returns (count, records) with
+    starts relative to ``text``; without ``out`` a count pass sizes it."""
+    _check_text(text)
+    if seg_off.dtype != torch.int64 or not seg_off.is_cuda or seg_off.dim() != 1 or seg_off.numel() < 1:
+        raise TypeError("seg_off must be a 1-D int64 CUDA tensor of n_seg + 1 offsets")
+    n_seg = seg_off.numel() - 1
+    L = lib()
+    res = torch.zeros(2, dtype=torch.int64, device=text.device)
+    s = _stream_ptr(stream)
+    tp = text.data_ptr() if text.numel() else None
+    if out is None:
+        _check(L.ac_match_segments(stt.handle, tp, seg_off.data_ptr(), n_seg, None, 0, res.data_ptr(), s))
+        out = torch.empty(max(1, int(res[0].item())), dtype=torch.int64, device=text.device)
+    _check(L.ac_match_segments(stt.handle, tp, seg_off.data_ptr(), n_seg, out.data_ptr(), out.numel(),
+                               res.data_ptr(), s))
     c, st = (int(x) for x in res.tolist())
     if st == AC_ERR_CAPACITY:
         raise CapacityError(st, f"{c} records do not fit in {out.numel()}", c)

@@ -415,6 +415,60 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     return rc;
 }
 
+// Packet batches (NEXT-2): independent segments, two passes (count, offsets,
+// emit) over one thread per segment.
+static ac_status match_segments(const ac_stt *h, const uint8_t *d_text, const uint64_t *d_seg_off, uint64_t n_seg,
+                                ac_match_t *d_out, uint64_t cap, ac_result *d_res, cudaStream_t stream) {
+    g_launches = 0;
+    if (!h || !d_res || (n_seg && (!d_seg_off || !d_text))) {
+        set_error("NULL stt, result, text or segment offsets");
+        return AC_ERR_INVALID_ARG;
+    }
+    AC_CUDA(cudaMemsetAsync(d_res, 0, sizeof(ac_result), stream), "memset result");
+    if (n_seg == 0 || h->host.n_patterns == 0) return AC_OK;
+    const SttView sg = view_of(h, 0);
+    const uint32_t tier = tier_of(h, sg), eb = h->host.entry_bytes;
+    const size_t smem = smem_of(h, sg);
+    ScanOut so{};
+    so.res = d_res;
+    so.out = reinterpret_cast<uint64_t *>(d_out);
+    auto note = [&](const char *name) {
+        if (g_launches < 16) g_names[g_launches] = name;
+        g_launches++;
+    };
+    if (!d_out) {
+        so.total = reinterpret_cast<unsigned long long *>(&d_res->count);
+        AC_CUDA(launch_segments(MODE_COUNT_TOTAL, eb, tier, d_text, d_seg_off, n_seg, sg, so, smem, stream),
+                "k_scan_segments(count)");
+        note("k_scan_segments(count)");
+        return AC_OK;
+    }
+    const size_t tiles = offsets_tiles(n_seg);
+    void *ws = nullptr;
+    AC_CUDA(cudaMallocAsync(&ws, n_seg * 16 + tiles * 8 + 16, stream), "cudaMallocAsync(workspace)");
+    uint64_t *counts = static_cast<uint64_t *>(ws);
+    uint64_t *chain_end = counts + n_seg;
+    uint64_t *tile_state = chain_end + n_seg;
+    unsigned int *counter = reinterpret_cast<unsigned int *>(tile_state + tiles);
+    so.chain_counts = counts;
+    so.chain_end = chain_end;
+    auto run = [&]() -> ac_status {
+        AC_CUDA(cudaMemsetAsync(tile_state, 0, tiles * 8 + 16, stream), "memset workspace");
+        AC_CUDA(launch_segments(MODE_COUNT_CHAINS, eb, tier, d_text, d_seg_off, n_seg, sg, so, smem, stream),
+                "k_scan_segments(count)");
+        note("k_scan_segments(count)");
+        AC_CUDA(launch_offsets(counts, n_seg, chain_end, tile_state, counter, d_res, cap, 1, stream), "k_offsets");
+        note("k_offsets");
+        AC_CUDA(launch_segments(MODE_EMIT, eb, tier, d_text, d_seg_off, n_seg, sg, so, smem, stream),
+                "k_scan_segments(emit)");
+        note("k_scan_segments(emit)");
+        return AC_OK;
+    };
+    const ac_status rc = run();
+    cudaFreeAsync(ws, stream);
+    return rc;
+}
+
 static ac_status finish_sync(ac_result *d_res, uint64_t *count, cudaStream_t stream) {
     ac_result hres;
     AC_CUDA(cudaMemcpyAsync(&hres, d_res, sizeof(hres), cudaMemcpyDeviceToHost, stream), "D2H result");
@@ -845,6 +899,16 @@ ac_status ac_match_async(const ac_stt *stt, const uint8_t *d_text, uint64_t n_ow
     try {
         return match_async(stt, d_text, n_owned, n_halo, base, d_out, cap, d_result,
                            static_cast<cudaStream_t>(stream), opts);
+    } catch (...) {
+        set_error("unexpected host exception");
+        return AC_ERR_NO_MEMORY;
+    }
+}
+
+ac_status ac_match_segments(const ac_stt *stt, const uint8_t *d_text, const uint64_t *d_seg_off, uint64_t n_seg,
+                            ac_match_t *d_out, uint64_t cap, ac_result *d_result, void *stream) {
+    try {
+        return match_segments(stt, d_text, d_seg_off, n_seg, d_out, cap, d_result, static_cast<cudaStream_t>(stream));
     } catch (...) {
         set_error("unexpected host exception");
         return AC_ERR_NO_MEMORY;

@@ -425,6 +425,38 @@ __global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ 
     }
 }
 
+// Packet batches (the NIDS workload of P:108): segment i
+// is text[seg_off[i], seg_off[i+1]) and is scanned from the start state on
+// its own -- no halo, no occurrence crosses a boundary.  One thread per
+// segment, right to left, so its records are canonical within the segment.
+template <typename E, int TIER, int MODE>
+__global__ void __launch_bounds__(GT) k_scan_segments(const uint8_t *__restrict__ text,
+                                                      const uint64_t *__restrict__ seg_off, uint64_t n_seg,
+                                                      SttView st, ScanOut so) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    uint8_t *s_cmap = smem;
+    E *s_stt = reinterpret_cast<E *>(smem + 256);
+    stage_tables<E>(s_cmap, s_stt, st);
+    __syncthreads();
+    if constexpr (MODE == MODE_EMIT) {
+        if (so.res->status != AC_OK) return;
+    }
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    uint32_t cnt = 0;
+    if (i < n_seg) {
+        const uint64_t lo = seg_off[i], hi = seg_off[i + 1];
+        uint64_t wp = 0;
+        if constexpr (MODE == MODE_EMIT) wp = so.chain_end[i];
+        uint32_t s = 0;
+        walk_global<E, TIER, MODE, true>(text, lo, hi, s, cnt, wp, s_cmap, s_stt, st, so);
+        if constexpr (MODE == MODE_COUNT_CHAINS) so.chain_counts[i] = cnt;
+    }
+    if constexpr (MODE == MODE_COUNT_TOTAL) {
+        const unsigned long long tot = warp_sum((unsigned long long)cnt);
+        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(so.total, tot);
+    }
+}
+
 // Re-scan the chains listed by k_gather (their matches overflowed the
 // scratch slot) straight into their final positions.  One CTA per listed
 // chain: the chain is split into GT sub-chains (each with its own halo
@@ -718,6 +750,43 @@ cudaError_t launch_global_tier(int mode, uint32_t eb, const uint8_t *text, uint6
         return with_mode(mode, [&](auto m) {
             return launch_global_m<uint32_t, TIER, decltype(m)::value>(text, n_total, st, a, b, so, smem, stream);
         });
+    }
+}
+
+template <typename E, int TIER, int MODE>
+static cudaError_t launch_segments_m(const uint8_t *text, const uint64_t *seg_off, uint64_t n_seg, const SttView &st,
+                                     const ScanOut &so, size_t smem, cudaStream_t stream) {
+    auto kern = k_scan_segments<E, TIER, MODE>;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    const unsigned grid = (unsigned)((n_seg + GT - 1) / GT);
+    if (grid == 0) return cudaSuccess;
+    kern<<<grid, GT, smem, stream>>>(text, seg_off, n_seg, st, so);
+    return cudaGetLastError();
+}
+
+template <typename E, int TIER>
+static cudaError_t launch_segments_e(int mode, const uint8_t *text, const uint64_t *seg_off, uint64_t n_seg,
+                                     const SttView &st, const ScanOut &so, size_t smem, cudaStream_t stream) {
+    switch (mode) {
+        case MODE_COUNT_TOTAL: return launch_segments_m<E, TIER, MODE_COUNT_TOTAL>(text, seg_off, n_seg, st, so, smem, stream);
+        case MODE_COUNT_CHAINS: return launch_segments_m<E, TIER, MODE_COUNT_CHAINS>(text, seg_off, n_seg, st, so, smem, stream);
+        case MODE_EMIT: return launch_segments_m<E, TIER, MODE_EMIT>(text, seg_off, n_seg, st, so, smem, stream);
+    }
+    return cudaErrorInvalidValue;
+}
+
+template <int TIER>
+cudaError_t launch_segments_tier(int mode, uint32_t eb, const uint8_t *text, const uint64_t *seg_off, uint64_t n_seg,
+                                 const SttView &st, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
+    const size_t smem = 256 + smem_stt;
+    if (eb == 2) return launch_segments_e<uint16_t, TIER>(mode, text, seg_off, n_seg, st, so, smem, stream);
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return cudaErrorInvalidValue;
+    } else {
+        return launch_segments_e<uint32_t, TIER>(mode, text, seg_off, n_seg, st, so, smem, stream);
     }
 }
 

@@ -155,6 +155,16 @@ cudaError_t launch_gather(const uint64_t *counts, const uint64_t *chain_end, uin
     return cudaGetLastError();
 }
 
+cudaError_t launch_segments(int mode, uint32_t eb, uint32_t tier, const uint8_t *text, const uint64_t *seg_off,
+                            uint64_t n_seg, const SttView &st, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
+    switch (tier) {
+        case AC_TIER_SMEM: return launch_segments_tier<AC_TIER_SMEM>(mode, eb, text, seg_off, n_seg, st, so, smem_stt, stream);
+        case AC_TIER_HYBRID: return launch_segments_tier<AC_TIER_HYBRID>(mode, eb, text, seg_off, n_seg, st, so, smem_stt, stream);
+        case AC_TIER_COMPACT: return launch_segments_tier<AC_TIER_COMPACT>(mode, eb, text, seg_off, n_seg, st, so, smem_stt, stream);
+        default: return launch_segments_tier<AC_TIER_GLOBAL>(mode, eb, text, seg_off, n_seg, st, so, smem_stt, stream);
+    }
+}
+
 cudaError_t launch_rewalk(uint32_t eb, uint32_t tier, const uint8_t *text, uint64_t n_total, const SttView &st,
                           const Region &a, const Region &b, const StagedGeom &g, const ScanOut &so,
                           const uint64_t *list, const unsigned int *list_n, size_t smem_stt, int num_sms,

@@ -118,6 +118,11 @@ cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtenso
                                const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
                                cudaStream_t stream);
 template <int TIER>
+cudaError_t launch_segments_tier(int mode, uint32_t eb, const uint8_t *text, const uint64_t *seg_off, uint64_t n_seg,
+                                 const SttView &st, const ScanOut &so, size_t smem_stt, cudaStream_t stream);
+cudaError_t launch_segments(int mode, uint32_t eb, uint32_t tier, const uint8_t *text, const uint64_t *seg_off,
+                            uint64_t n_seg, const SttView &st, const ScanOut &so, size_t smem_stt, cudaStream_t stream);
+template <int TIER>
 cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_total, const SttView &st,
                                const Region &a, const Region &b, const StagedGeom &g, const ScanOut &so,
                                const uint64_t *list, const unsigned int *list_n, size_t smem_stt, int num_sms,

@@ -16,3 +16,8 @@ template cudaError_t launch_rewalk_tier<AC_TIER_COMPACT>(uint32_t, const uint8_t
                                                      const ScanOut &, const uint64_t *, const unsigned int *, size_t,
                                                      int, cudaStream_t);
 }  // namespace acx
+
+namespace acx {
+template cudaError_t launch_segments_tier<AC_TIER_COMPACT>(int, uint32_t, const uint8_t *, const uint64_t *, uint64_t,
+                                                       const SttView &, const ScanOut &, size_t, cudaStream_t);
+}  // namespace acx

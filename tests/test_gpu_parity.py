@@ -390,6 +390,29 @@ def test_host_entry_point_pipelined_chunks():
     assert e.value.count == want.size
 
 
+@pytest.mark.parametrize("name", ["c3", "c2"])
+def test_packet_segments(name):
+    """NEXT-2 packet batches: every segment scanned on its own."""
+    w = synth.make(name, n=(1 << 20) + 13)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    rng = np.random.default_rng(5)
+    cuts = np.unique(np.concatenate([[0, w.text.size], rng.integers(0, w.text.size, size=900),
+                                     rng.integers(0, 64, size=5)]))  # includes empty-ish and tiny segments
+    parts = []
+    for lo, hi in zip(cuts[:-1].tolist(), cuts[1:].tolist()):
+        parts.append(oracle_keys(o, w.text[lo:hi]) + (lo << 24))
+    want = np.concatenate(parts)
+    t = torch.from_numpy(w.text).cuda()
+    seg = torch.from_numpy(cuts.astype(np.int64)).cuda()
+    c, recs = ac.match_segments(stt, t, seg)
+    assert c == want.size
+    assert_same(recs.cpu().numpy(), want)
+    # segments == [0, n) is the plain scan
+    c1, r1 = ac.match_segments(stt, t, torch.tensor([0, t.numel()], dtype=torch.int64, device="cuda"))
+    assert_same(r1.cpu().numpy(), oracle_keys(o, w.text))
+
+
 def test_determinism():
     w = synth.make("c2", n=(2 << 20) + 1, n_patterns=500)
     stt = ac.build(w.patterns)
