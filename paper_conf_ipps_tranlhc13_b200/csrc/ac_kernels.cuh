@@ -669,7 +669,39 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                     v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
                     kb[k] = (so.base + g.m0 + cbase[k] + col0 + q * 16) << 24;
                 }
-                if constexpr (STRIDE == 2) {
+                if constexpr (STRIDE == 1 && K == 1 && sizeof(E) == 2) {
+                    // Deferred emission: walk the 16 bytes recording the
+                    // flag bits and the (16-bit) states in registers, then
+                    // emit in a warp-uniform loop that runs max-over-lanes
+                    // popcount times (~3 for C2) instead of 16 times.
+                    uint32_t hist[8], fm = 0, st0 = s[0];
+#pragma unroll
+                    for (int bb = 15; bb >= 0; --bb) {
+                        const uint32_t e = next_entry<E, TIER>(s_stt, st, st0, s_cmap[byte_of(v[0], bb)]);
+                        st0 = e & EntryBits<E>::MASK;
+                        fm |= ((e >> 15) & 1u) << bb;
+                        if (bb & 1)
+                            hist[bb >> 1] = st0;
+                        else
+                            hist[bb >> 1] |= st0 << 16;
+                    }
+                    s[0] = st0;
+                    if (!live[0]) fm = 0;
+                    while (__any_sync(0xffffffffu, fm)) {
+                        if (fm) {
+                            const int bb = 31 - __clz(fm);
+                            fm &= ~(1u << bb);
+                            const int i = bb >> 1;
+                            const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
+                            const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
+                            const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
+                            const uint32_t pr = (i & 4) ? b1 : b0;
+                            const uint32_t x = (bb & 1) ? (pr & 0xFFFFu) : (pr >> 16);
+                            emit_outputs<E, TIER, MODE>(x, kb[0] + ((uint64_t)bb << 24), cnt[0], wp[0], s_stt, st,
+                                                        so);
+                        }
+                    }
+                } else if constexpr (STRIDE == 2) {
 #pragma unroll
                     for (int bb = 15; bb >= 1; bb -= 2) {
 #pragma unroll
