@@ -669,7 +669,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                     v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
                     kb[k] = (so.base + g.m0 + cbase[k] + col0 + q * 16) << 24;
                 }
-                if constexpr (STRIDE == 1 && K == 1 && sizeof(E) == 2) {
+                // (COMPACT counting keeps its predicated per-byte count: measured faster)
+                constexpr bool kDeferred = STRIDE == 1 && K == 1 && sizeof(E) == 2 &&
+                                           (TIER != AC_TIER_COMPACT || MODE == MODE_EMIT || MODE == MODE_EMIT_OPT);
+                if constexpr (kDeferred) {
                     // Deferred emission: walk the 16 bytes recording the
                     // flag bits and the (16-bit) states in registers, then
                     // emit in a warp-uniform loop that runs max-over-lanes
