@@ -40,7 +40,10 @@ static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slot
 // COMPACT budget used by ac_compile (no device): B200's 227 KB opt-in shared
 // memory minus the lean staged variant's ring and bookkeeping (= stt_budget)
 #define kDefaultCompactBudget (232448 - staged_smem_bytes(staged_variant(kLeanVariant), 0) - 1024)
-static const uint64_t kStagedMinBytes = 64 * 1024;
+// Below ~32 MiB the staged kernel cannot fill 148 SMs x 1024 chains with
+// chains of >= 256 B; the global kernel's shorter chains win (C1: 1 MiB list
+// 0.037 ms global vs 0.052 ms staged).
+static const uint64_t kStagedMinBytes = 32ull << 20;
 static const uint64_t kStagedMinChain = 256;
 
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda).
