@@ -60,6 +60,19 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     return fn;
 }
 
+// Makes `device` current for the scope of a call and restores the caller's.
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int device) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != device) cudaSetDevice(device);
+        else prev = -1;
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
 // Per-thread, per-device side stream + fork/join events (created lazily,
 // kept for the thread's lifetime).
 struct SideStream {
@@ -899,6 +912,11 @@ ac_status ac_stt_pattern_lengths(const ac_stt *h, uint32_t *lens) {
 ac_status ac_match_async(const ac_stt *stt, const uint8_t *d_text, uint64_t n_owned, uint64_t n_halo, uint64_t base,
                          ac_match_t *d_out, uint64_t cap, ac_result *d_result, void *stream,
                          const ac_match_opts *opts) {
+    if (!stt) {
+        set_error("stt is NULL");
+        return AC_ERR_INVALID_ARG;
+    }
+    DeviceGuard guard(stt->device);  // launches go to the STT's device
     try {
         return match_async(stt, d_text, n_owned, n_halo, base, d_out, cap, d_result,
                            static_cast<cudaStream_t>(stream), opts);
@@ -910,6 +928,11 @@ ac_status ac_match_async(const ac_stt *stt, const uint8_t *d_text, uint64_t n_ow
 
 ac_status ac_match_segments(const ac_stt *stt, const uint8_t *d_text, const uint64_t *d_seg_off, uint64_t n_seg,
                             ac_match_t *d_out, uint64_t cap, ac_result *d_result, void *stream) {
+    if (!stt) {
+        set_error("stt is NULL");
+        return AC_ERR_INVALID_ARG;
+    }
+    DeviceGuard guard(stt->device);
     try {
         return match_segments(stt, d_text, d_seg_off, n_seg, d_out, cap, d_result, static_cast<cudaStream_t>(stream));
     } catch (...) {
