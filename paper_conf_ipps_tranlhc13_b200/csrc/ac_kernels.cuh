@@ -672,7 +672,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                 // (COMPACT counting keeps its predicated per-byte count: measured faster)
                 constexpr bool kDeferred = STRIDE == 1 && K == 1 && sizeof(E) == 2 &&
                                            (TIER != AC_TIER_COMPACT || MODE == MODE_EMIT || MODE == MODE_EMIT_OPT);
-                constexpr bool kRewalk = STRIDE == 1 && K == 1 && sizeof(E) == 4;
+                // Deferred-by-rewalk for 32-bit tables: measured SLOWER on C3
+                // (count 3.81 -> 4.95 ms, the L1-bound walk lost its overlap),
+                // so it is compiled out; kept for the record and for experiments.
+                constexpr bool kRewalk = false && STRIDE == 1 && K == 1 && sizeof(E) == 4;
                 if constexpr (kRewalk) {
                     // 32-bit states do not pack into a register history: walk
                     // the chunk recording only the flag mask, and re-walk it
