@@ -706,16 +706,16 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                     // flag bits and the (16-bit) states in registers, then
                     // emit in a warp-uniform loop that runs max-over-lanes
                     // popcount times (~3 for C2) instead of 16 times.
-                    uint32_t hist[8], fm = 0, st0 = s[0];
+                    uint32_t hist[8], fm = 0, st0 = s[0], odd = 0;
 #pragma unroll
                     for (int bb = 15; bb >= 0; --bb) {
                         const uint32_t e = next_entry<E, TIER>(s_stt, st, st0, s_cmap[byte_of(v[0], bb)]);
                         st0 = e & EntryBits<E>::MASK;
-                        fm |= ((e >> 15) & 1u) << bb;
+                        fm = (fm << 1) | (e >> 15);  // byte bb's flag ends at bit bb
                         if (bb & 1)
-                            hist[bb >> 1] = st0;
+                            odd = st0;
                         else
-                            hist[bb >> 1] |= st0 << 16;
+                            hist[bb >> 1] = __byte_perm(odd, st0, 0x5410);  // (odd, even << 16)
                     }
                     s[0] = st0;
                     if (!live[0]) fm = 0;
