@@ -109,18 +109,20 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
     const uint32_t sp = s >= st.c_dense;
     const uint32_t ad = base + ((s * st.c_dstride + cls) << 1);
     const uint32_t as = base + st.c_sparse_off + ((s - st.c_dense) << 3);
-    uint32_t lo = 0, hi = 0;
+    // Outputs are write-only ("=r"): hi is read only when sp, e3 only when
+    // need, so the predicated-off lanes' stale values are never used.
+    uint32_t lo, hi;
     asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t"
         "@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t"
         "@!p ld.shared.u16 %0, [%4];\n\t}"
-        : "+r"(lo), "+r"(hi)
+        : "=r"(lo), "=r"(hi)
         : "r"(as), "r"(sp), "r"(ad));
     const uint32_t h1 = ((lo >> 16) & 0xFFu) == cls, h2 = (lo >> 24) == cls;
     const uint32_t need = sp & (1u ^ (h1 | h2));  // sparse and no exception hit
     const uint32_t ad2 = base + (((lo & 0xFFFFu) * st.c_dstride + cls) << 1);
-    uint32_t e3 = 0;
+    uint32_t e3;
     asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u16 %0, [%1];\n\t}"
-        : "+r"(e3)
+        : "=r"(e3)
         : "r"(ad2), "r"(need));
     const uint32_t ex = h1 ? (hi & 0xFFFFu) : (hi >> 16);
     return sp ? (need ? e3 : ex) : lo;
@@ -564,8 +566,11 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     k_scan_staged(const __grid_constant__ CUtensorMap tmap, const uint8_t *__restrict__ mtext, SttView st,
                   StagedGeom g, ScanOut so) {
     using Sh = StagedShape<WARPS, K, W, NST, SWIZZLE>;
-    extern __shared__ uint8_t smem_raw[];
-    uint8_t *ring = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    // Swizzled tiles need their 1024-B atom alignment at run time; unswizzled
+    // (W = 16) tiles only need TMA's 128 B, which the dynamic base has, so the
+    // whole layout -- and the STT base -- is a compile-time constant.
+    uint8_t *ring = Sh::SWZ ? smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u) : smem_raw;
     uint64_t *bars = reinterpret_cast<uint64_t *>(ring + Sh::RING);
     uint8_t *s_cmap = ring + Sh::RING + Sh::BARS;
     E *s_stt = reinterpret_cast<E *>(s_cmap + 256);
