@@ -141,7 +141,17 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
         }
         const uint64_t *src = scratch + c * q + (q - cnt);
         uint64_t *dst = out + chain_end[c] - cnt;
-        for (uint64_t i = lane; i < cnt; i += 32) dst[i] = __ldg(src + i);
+        // four records in flight per lane before the stores
+        uint64_t i = lane;
+        for (; i + 96 < cnt; i += 128) {
+            const uint64_t a = __ldg(src + i), b = __ldg(src + i + 32), d = __ldg(src + i + 64),
+                           e = __ldg(src + i + 96);
+            dst[i] = a;
+            dst[i + 32] = b;
+            dst[i + 64] = d;
+            dst[i + 96] = e;
+        }
+        for (; i < cnt; i += 32) dst[i] = __ldg(src + i);
     }
 }
 
