@@ -122,8 +122,11 @@ typedef struct {
      * [sparse records at compact_sparse_off: (n_states - compact_dense) x 8 B,
      *  lo32 = fd | c1 << 16 | c2 << 24, hi32 = t1 | t2 << 16]
      * [output table at compact_out_off: (compact_od + compact_os) x
-     *  (u32 payload, u32 count)], compact ids: 0 = root, then dense output
-     * states, other dense, sparse output states, other sparse.           */
+     *  (u32 payload, u32 count)], compact ids: 0 = root, then other dense
+     * states, dense output states, sparse output states, other sparse: the
+     * output states are ids [compact_dense - compact_od, compact_dense +
+     * compact_os) and the output slot of id x is x - (compact_dense -
+     * compact_od).                                                      */
     uint32_t compact_dense, compact_od, compact_os, compact_dstride;
     uint32_t compact_sparse_off, compact_out_off;
     uint64_t compact_bytes;

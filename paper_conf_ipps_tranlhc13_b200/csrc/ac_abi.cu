@@ -156,10 +156,9 @@ static SttView view_of(const ac_stt *h, int v) {
     s.halo = h->host.maxlen ? h->host.maxlen - 1 : 0;
     s.info_col = h->host.info_col;
     s.c_dense = h->host.c_dense;
-    s.c_od = h->host.c_od;
-    s.c_dstride = h->host.c_dstride;
-    s.c_sparse_off = h->host.c_sparse_off;
-    s.c_out_off = h->host.c_out_off;
+    s.c_row_bytes = 2 * h->host.c_dstride;
+    s.c_sparse_x0 = h->host.c_sparse_off - 8u * h->host.c_dense;
+    s.c_out_x0 = h->host.c_out_off - 8u * (h->host.c_dense - h->host.c_od);
     s.stt2 = v ? h->d_stt2 : nullptr;  // only the staged kernel walks two bytes per lookup
     s.stride2 = h->host.stride2;
     s.n_classes = h->host.n_classes;

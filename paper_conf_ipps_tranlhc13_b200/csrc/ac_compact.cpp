@@ -15,10 +15,10 @@
 //     -- exactly the classes where delta(s,.) differs from delta(fd(s),.).
 //     delta(s,c) = exception if c matches one, else dense[fd(s)][c]: at most
 //     two shared-memory loads per byte, no loop.
-//   * Output states are numbered first inside each group so the output
-//     table index is arithmetic: oidx = x - 1 (dense, x >= 1) or
-//     c_od + x - c_dense (sparse); each table slot holds (payload, count)
-//     exactly like the dense rows' output summary.
+//   * Output states are numbered last among the dense and first among the
+//     sparse states, so their ids are contiguous and the output table index
+//     is one subtraction: oidx = x - (c_dense - c_od); each table slot holds
+//     (payload, count) exactly like the dense rows' output summary.
 //
 // Entries keep the dense layout's convention: bit 15 = output(next) != {},
 // bits 0..14 = next state (COMPACT requires <= 32768 states and C <= 255).
@@ -83,15 +83,17 @@ bool compact_table(ac_table &t, size_t budget) {
         return e;
     };
     auto is_out = [&](uint32_t s) { return t.out_off[s + 1] > t.out_off[s]; };
-    // numbering: root, dense outputs, other dense, sparse outputs, other sparse
+    // numbering: root, other dense, dense outputs, sparse outputs, other
+    // sparse -- the output states form ONE contiguous id range
+    // [c_dense - c_od, c_dense + c_os), so oidx = x - (c_dense - c_od)
     std::vector<uint32_t> perm;  // compact id -> BFS id
     perm.reserve(S);
     perm.push_back(0);
     uint32_t od = 0, os = 0;
     for (uint32_t s = 1; s < S; s++)
-        if (dense[s] && is_out(s)) perm.push_back(s), od++;
-    for (uint32_t s = 1; s < S; s++)
         if (dense[s] && !is_out(s)) perm.push_back(s);
+    for (uint32_t s = 1; s < S; s++)
+        if (dense[s] && is_out(s)) perm.push_back(s), od++;
     for (uint32_t s = 1; s < S; s++)
         if (!dense[s] && is_out(s)) perm.push_back(s), os++;
     for (uint32_t s = 1; s < S; s++)
@@ -143,8 +145,7 @@ bool compact_table(ac_table &t, size_t budget) {
         std::memcpy(&blob[out_base + (size_t)oidx * 8], &payload, 4);
         std::memcpy(&blob[out_base + (size_t)oidx * 8 + 4], &count, 4);
     };
-    for (uint32_t i = 0; i < od; i++) put_out(i, perm[1 + i]);
-    for (uint32_t i = 0; i < os; i++) put_out(od + i, perm[nd + i]);
+    for (uint32_t i = 0; i < od + os; i++) put_out(i, perm[nd - od + i]);
 
     t.compact.swap(blob);
     t.c_perm.swap(perm);

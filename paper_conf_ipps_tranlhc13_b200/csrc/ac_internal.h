@@ -28,9 +28,9 @@ struct ac_table {
 
     // COMPACT encoding, built by compact_table():
     //   [dense rows: c_dense x c_dstride u16][sparse records: (S - c_dense) x 8 B][output table: n_out x 8 B]
-    // in its own numbering: 0 = root, [1, 1 + c_od) = dense output states,
-    // then the other dense states, [c_dense, c_dense + c_os) = sparse output
-    // states, then the other sparse states.
+    // in its own numbering: 0 = root, then the other dense states,
+    // [c_dense - c_od, c_dense) = dense output states, [c_dense, c_dense +
+    // c_os) = sparse output states, then the other sparse states.
     uint32_t c_dense = 0, c_od = 0, c_os = 0, c_dstride = 0;
     uint32_t c_sparse_off = 0, c_out_off = 0;  // byte offsets inside `compact`
     std::vector<uint8_t> compact;

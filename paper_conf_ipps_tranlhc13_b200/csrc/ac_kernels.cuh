@@ -105,26 +105,28 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
 // COMPACT: a dense row, or a sparse record's exception, or the dense row of
 // the record's default state fd(s) -- at most two shared-memory loads, issued
 // as predicated loads so lanes in dense and sparse states never diverge.
+// (Each predicated load's destination register is pre-loaded with a value
+// that is dead afterwards -- its own address -- so no zeroing moves are
+// needed; write-only "=r" outputs made ptxas spill 372 B per thread.)
 __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
     const uint32_t sp = s >= st.c_dense;
-    const uint32_t ad = base + ((s * st.c_dstride + cls) << 1);
-    const uint32_t as = base + st.c_sparse_off + ((s - st.c_dense) << 3);
-    // ("+r" with zero-initialised outputs: write-only "=r" outputs on the
-    //  predicated loads made ptxas spill 372 B per thread -- measured 1.5x slower)
-    uint32_t lo = 0, hi = 0;
-    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t"
-        "@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t"
-        "@!p ld.shared.u16 %0, [%4];\n\t}"
+    const uint32_t cb = base + (cls << 1);             // column cls of row 0
+    uint32_t lo = base + st.c_sparse_x0 + (s << 3);    // sparse record of s (garbage if dense)
+    uint32_t hi = cb + s * st.c_row_bytes;             // dense entry (s, cls) (garbage if sparse)
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t"
+        "@p ld.shared.v2.u32 {%0, %1}, [%0];\n\t"
+        "@!p ld.shared.u16 %0, [%1];\n\t}"
         : "+r"(lo), "+r"(hi)
-        : "r"(as), "r"(sp), "r"(ad));
-    const uint32_t h1 = ((lo >> 16) & 0xFFu) == cls, h2 = (lo >> 24) == cls;
-    const uint32_t need = sp & (1u ^ (h1 | h2));  // sparse and no exception hit
-    const uint32_t ad2 = base + (((lo & 0xFFFFu) * st.c_dstride + cls) << 1);
-    uint32_t e3 = 0;
-    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.u16 %0, [%1];\n\t}"
+        : "r"(sp));
+    // sparse: lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
+    const uint32_t x = lo ^ __byte_perm(cls, 0, 0x0000);  // byte k of x is 0 iff byte k of lo == cls
+    const uint32_t h1 = (x & 0x00FF0000u) == 0, h2 = (x & 0xFF000000u) == 0;
+    const uint32_t need = sp & (1u ^ (h1 | h2));           // sparse and no exception hit
+    uint32_t e3 = cb + (lo & 0xFFFFu) * st.c_row_bytes;    // dense entry (fd, cls)
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
         : "+r"(e3)
-        : "r"(ad2), "r"(need));
-    const uint32_t ex = h1 ? (hi & 0xFFFFu) : (hi >> 16);
+        : "r"(need));
+    const uint32_t ex = __byte_perm(hi, 0, h1 ? 0x4410 : 0x4432);
     return sp ? (need ? e3 : ex) : lo;
 }
 
@@ -147,8 +149,7 @@ __device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uin
 // COMPACT output table slot of output state s: (payload, count).
 template <typename E>
 __device__ __forceinline__ uint2 compact_out(const E *s_stt, const SttView &st, uint32_t s) {
-    const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
-    return reinterpret_cast<const uint2 *>(reinterpret_cast<const uint8_t *>(s_stt) + st.c_out_off)[oidx];
+    return *reinterpret_cast<const uint2 *>(reinterpret_cast<const uint8_t *>(s_stt) + (st.c_out_x0 + (s << 3)));
 }
 
 // Output summary of state s, stored in the padding of its own STT row
@@ -185,14 +186,24 @@ __device__ __forceinline__ uint32_t out_payload(const E *s_stt, const SttView &s
     }
 }
 
+// (payload, count) of output state s through its tier; a saturated 16-bit
+// count falls back to the CSR offsets.
+template <typename E, int TIER>
+__device__ __forceinline__ uint2 compact_or_row_out(const E *s_stt, const SttView &st, uint32_t s) {
+    if constexpr (TIER == AC_TIER_COMPACT) {
+        return compact_out<E>(s_stt, st, s);
+    } else {
+        return make_uint2(out_payload<E, TIER>(s_stt, st, s), out_count<E, TIER>(s_stt, st, s));
+    }
+}
+
 // (payload, count) of state s if f != 0, else (0, 0) -- predicated loads
 // through the state's residency tier, so lanes never branch on a match.
 template <typename E, int TIER, bool PAYLOAD>
 __device__ __forceinline__ uint2 out_info_pred(const E *s_stt, const SttView &st, uint32_t s, uint32_t f) {
     uint32_t pay = 0, c = 0;
     if constexpr (TIER == AC_TIER_COMPACT) {
-        const uint32_t oidx = s < st.c_dense ? s - 1 : st.c_od + s - st.c_dense;
-        const uint32_t a = smem_u32(s_stt) + st.c_out_off + (oidx << 3);
+        const uint32_t a = smem_u32(s_stt) + st.c_out_x0 + (s << 3);
         asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t}"
             : "+r"(pay), "+r"(c)
             : "r"(a), "r"(f));
@@ -351,9 +362,19 @@ __device__ __forceinline__ void ac_step2(uint32_t &s, uint32_t &cnt, uint64_t &w
     s = e & T2_MASK;
 }
 
+// Predicated 8-byte global store to base[k] (k signed; one IMAD.WIDE for
+// the address, no branch around the store).
+__device__ __forceinline__ void st_global_if(const uint64_t *base, int32_t k, uint64_t v, bool pred) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ne.u32 p, %3, 0;\n\t"
+        "mad.wide.s32 a, %1, 8, %0;\n\t@p st.global.u64 [a], %2;\n\t}" ::"l"(base),
+        "r"(k), "l"(v), "r"((uint32_t)pred)
+        : "memory");
+}
+
 __device__ __forceinline__ uint32_t byte_of(const uint4 &v, int bb) {
     const uint32_t w = (bb >> 2) == 0 ? v.x : (bb >> 2) == 1 ? v.y : (bb >> 2) == 2 ? v.z : v.w;
-    return (w >> (8 * (bb & 3))) & 0xffu;
+    return __byte_perm(w, 0, 0x4440 | (bb & 3));  // one PRMT: zero-extended byte bb & 3
 }
 
 __device__ __forceinline__ unsigned long long warp_sum(unsigned long long v) {
@@ -724,6 +745,38 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                     }
                     s[0] = st0;
                     if (!live[0]) fm = 0;
+                    if constexpr (MODE == MODE_EMIT_OPT) {
+                        // record k of the chain goes to slot last - k (if k < q);
+                        // nk = -k keeps the address one IMAD.WIDE away
+                        const uint64_t *const last = reinterpret_cast<const uint64_t *>(wp[0]);
+                        int32_t nk = -(int32_t)cnt[0];
+                        const int32_t nq = -(int32_t)so.q;
+                        while (__any_sync(0xffffffffu, fm)) {
+                            if (fm) {
+                                const int bb = 31 - __clz(fm);
+                                fm ^= 1u << bb;
+                                const int i = bb >> 1;
+                                const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
+                                const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
+                                const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
+                                const uint32_t pr = (i & 4) ? b1 : b0;
+                                const uint32_t x = __byte_perm(pr, 0, (bb & 1) ? 0x4410 : 0x4432);
+                                const uint2 o = compact_or_row_out<E, TIER>(s_stt, st, x);
+                                // key = (start << 24) | pid, start = chunk start + bb (pid < 2^24)
+                                const uint32_t kl = (uint32_t)bb << 24;
+                                if (o.y == 1) {
+                                    st_global_if(last, nk, kb[0] + (kl | o.x), nk > nq);
+                                    --nk;
+                                } else {
+                                    for (uint32_t j = o.x + o.y; j > o.x; --j) {
+                                        st_global_if(last, nk, kb[0] + (kl | __ldg(st.out_ids + j - 1)), nk > nq);
+                                        --nk;
+                                    }
+                                }
+                            }
+                        }
+                        cnt[0] = (uint32_t)(-nk);
+                    } else
                     while (__any_sync(0xffffffffu, fm)) {
                         if (fm) {
                             const int bb = 31 - __clz(fm);

@@ -28,8 +28,12 @@ struct SttView {
     uint32_t halo;            // maxlen - 1
     uint32_t info_col;        // entry index of the row's output summary (payload u32, count)
     uint32_t smem_bytes;      // STT bytes staged into shared memory
-    // COMPACT tier (ac_compact.cpp): dense/sparse split and blob offsets
-    uint32_t c_dense, c_od, c_dstride, c_sparse_off, c_out_off;
+    // COMPACT tier (ac_compact.cpp): the dense/sparse split and byte offsets
+    // inside the blob, pre-biased so that each address is one multiply-add
+    // of the compact id x: dense row x at x * c_row_bytes, sparse record x at
+    // c_sparse_x0 + 8 x, output slot of output state x at c_out_x0 + 8 x
+    // (both x0 wrap around modulo 2^32 on purpose)
+    uint32_t c_dense, c_row_bytes, c_sparse_x0, c_out_x0;
     // two-byte table (NEXT-4): row s, column c1 * n_classes + c2; NULL = off
     const uint32_t *stt2;
     uint32_t stride2, n_classes;

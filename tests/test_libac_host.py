@@ -186,12 +186,12 @@ def test_compact_encoding_equals_dense(which):
     # output-state numbering and the output table
     nd, od, os_ = d["compact_dense"], d["compact_od"], d["compact_os"]
     has_out = np.diff(t.out_off.astype(np.int64))[perm] > 0
-    assert has_out[1:1 + od].all() and not has_out[1 + od:nd].any()
-    assert has_out[nd:nd + os_].all() and not has_out[nd + os_:].any() and not has_out[0]
-    for x in list(range(1, 1 + od)) + list(range(nd, nd + os_)):
+    # output states are exactly the contiguous ids [nd - od, nd + os)
+    assert has_out[nd - od:nd + os_].all() and not has_out[:nd - od].any() and not has_out[nd + os_:].any()
+    for x in range(nd - od, nd + os_):
         s = perm[x]
         outs = t.out_ids[t.out_off[s]:t.out_off[s + 1]].tolist()
-        oidx = x - 1 if x < nd else od + x - nd
+        oidx = x - (nd - od)
         payload, count = ot[oidx].tolist()
         assert count == len(outs) and payload == (outs[0] if count == 1 else int(t.out_off[s]))
     assert d["compact_bytes"] <= 232448 - (1024 + 32 * 2 * 512 + 512 + 256) - 1024
