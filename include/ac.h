@@ -79,7 +79,7 @@ typedef struct ac_table ac_table;
  * prefix in shared memory, the rest through L1/L2.  GLOBAL: L1/L2 only.
  * COMPACT: dense rows for shallow states + 8-byte default-transition records
  * for the others + an output table, all in shared memory (<= 32768 states,
- * <= 255 classes).  AUTO = SMEM if the dense table
+ * <= 127 classes).  AUTO = SMEM if the dense table
  * fits, else COMPACT if that fits, else GLOBAL. */
 enum { AC_TIER_AUTO = 0, AC_TIER_SMEM = 1, AC_TIER_HYBRID = 2, AC_TIER_GLOBAL = 3, AC_TIER_COMPACT = 4 };
 
@@ -120,7 +120,8 @@ typedef struct {
     /* COMPACT encoding (valid when compact_bytes != 0): byte layout
      * [dense rows: compact_dense x compact_dstride u16]
      * [sparse records at compact_sparse_off: (n_states - compact_dense) x 8 B,
-     *  lo32 = fd | c1 << 16 | c2 << 24, hi32 = t1 | t2 << 16]
+     *  lo32 = fd | 2 c1 << 16 | 2 c2 << 24 (doubled classes, 0xFF = none),
+     *  hi32 = t1 | t2 << 16]
      * [output table at compact_out_off: (compact_od + compact_os) x
      *  (u32 payload, u32 count)], compact ids: 0 = root, then other dense
      * states, dense output states, sparse output states, other sparse: the

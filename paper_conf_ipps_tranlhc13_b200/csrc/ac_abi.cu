@@ -864,7 +864,9 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             return fail(e, "H2D stt2");
     }
     if ((e = cudaMalloc(&h->d_class_map, 256)) != cudaSuccess) return fail(e, "cudaMalloc(class map)");
-    if ((e = cudaMemcpy(h->d_class_map, t.class_map, 256, cudaMemcpyHostToDevice)) != cudaSuccess)
+    uint8_t cmap[256];  // COMPACT walks with doubled classes (column byte offsets)
+    for (int b = 0; b < 256; b++) cmap[b] = tier == AC_TIER_COMPACT ? (uint8_t)(2 * t.class_map[b]) : t.class_map[b];
+    if ((e = cudaMemcpy(h->d_class_map, cmap, 256, cudaMemcpyHostToDevice)) != cudaSuccess)
         return fail(e, "H2D class map");
     if ((e = cudaMalloc(&h->d_out_off, t.out_off.size() * 4)) != cudaSuccess) return fail(e, "cudaMalloc(out_off)");
     if ((e = cudaMemcpy(h->d_out_off, t.out_off.data(), t.out_off.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)

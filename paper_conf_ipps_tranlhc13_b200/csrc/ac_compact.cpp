@@ -21,7 +21,10 @@
 //     (payload, count) exactly like the dense rows' output summary.
 //
 // Entries keep the dense layout's convention: bit 15 = output(next) != {},
-// bits 0..14 = next state (COMPACT requires <= 32768 states and C <= 255).
+// bits 0..14 = next state (COMPACT requires <= 32768 states and C <= 127).
+// The device class map of a COMPACT automaton holds 2 x class: the byte
+// offset of the class's column inside a dense row, compared directly with
+// the records' (doubled) exception classes.
 #include <algorithm>
 #include <cstring>
 
@@ -65,7 +68,7 @@ size_t compact_bytes_for(const ac_table &t, uint32_t d, std::vector<uint8_t> *de
 // Returns false (t unchanged) when the automaton cannot be compacted.
 bool compact_table(ac_table &t, size_t budget) {
     const uint32_t S = t.n_states, C = t.n_classes, stride = t.row_stride;
-    if (t.entry_bytes != 2 || S > 32768 || C > 255 || S == 0) return false;
+    if (t.entry_bytes != 2 || S > 32768 || C > 127 || S == 0) return false;
     uint32_t maxd = 0;
     for (uint32_t s = 0; s < S; s++) maxd = std::max(maxd, t.depth[s]);
     // the deepest dense prefix that fits (the size is not monotonic in d:
@@ -114,7 +117,9 @@ bool compact_table(ac_table &t, size_t budget) {
             std::memcpy(&blob[((size_t)x * dstride + c) * 2], &e, 2);
         }
     }
-    // sparse records: lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
+    // sparse records: lo = fd | 2 c1 << 16 | 2 c2 << 24, hi = t1 | t2 << 16
+    // (classes doubled, as in the COMPACT class map: a doubled class is the
+    // byte offset of its column in a dense row; 0xFF = no exception)
     std::vector<uint32_t> fd(S, 0);
     for (uint32_t s = 1; s < S; s++)
         if (!dense[s]) fd[s] = dense[t.fail[s]] ? t.fail[s] : fd[t.fail[s]];
@@ -126,7 +131,7 @@ bool compact_table(ac_table &t, size_t budget) {
         for (uint32_t c = 0; c < C; c++) {
             const uint16_t e = delta_e(s, c);
             if ((e & 0x7fffu) != (delta_e(fd[s], c) & 0x7fffu)) {
-                cls[k] = c;
+                cls[k] = 2 * c;
                 tgt[k] = enc(e);
                 k++;
             }

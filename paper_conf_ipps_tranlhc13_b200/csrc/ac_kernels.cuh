@@ -108,24 +108,27 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
 // (Each predicated load's destination register is pre-loaded with a value
 // that is dead afterwards -- its own address -- so no zeroing moves are
 // needed; write-only "=r" outputs made ptxas spill 372 B per thread.)
-__device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
+__device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls2) {
+    // cls2 = 2 x class (the COMPACT class map is pre-doubled): the byte
+    // offset of column cls inside a dense row, and the form in which the
+    // sparse records store their exception classes
     const uint32_t sp = s >= st.c_dense;
-    const uint32_t cb = base + (cls << 1);             // column cls of row 0
-    uint32_t lo = base + st.c_sparse_x0 + (s << 3);    // sparse record of s (garbage if dense)
-    uint32_t hi = cb + s * st.c_row_bytes;             // dense entry (s, cls) (garbage if sparse)
-    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t"
+    uint32_t lo, hi = cls2 + s * st.c_row_bytes;  // dense entry (s, cls) (garbage if sparse)
+    asm("mad.lo.u32 %0, %1, 8, %2;" : "=r"(lo) : "r"(s), "r"(base + st.c_sparse_x0));  // sparse record of s
+    asm("{\n\t.reg .pred p;\n\t.reg .u32 a;\n\tsetp.ne.u32 p, %2, 0;\n\t"
+        "add.u32 a, %1, %3;\n\t"
         "@p ld.shared.v2.u32 {%0, %1}, [%0];\n\t"
-        "@!p ld.shared.u16 %0, [%1];\n\t}"
+        "@!p ld.shared.u16 %0, [a];\n\t}"
         : "+r"(lo), "+r"(hi)
-        : "r"(sp));
-    // sparse: lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
-    const uint32_t x = lo ^ __byte_perm(cls, 0, 0x0000);  // byte k of x is 0 iff byte k of lo == cls
+        : "r"(sp), "r"(base));
+    // sparse: lo = fd | c1 << 16 | c2 << 24 (exception classes doubled), hi = t1 | t2 << 16
+    const uint32_t x = lo ^ __byte_perm(cls2, 0, 0x0000);  // byte k of x is 0 iff byte k of lo == cls2
     const uint32_t h1 = (x & 0x00FF0000u) == 0, h2 = (x & 0xFF000000u) == 0;
-    const uint32_t need = sp & (1u ^ (h1 | h2));           // sparse and no exception hit
-    uint32_t e3 = cb + (lo & 0xFFFFu) * st.c_row_bytes;    // dense entry (fd, cls)
-    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
+    const uint32_t need = sp & (1u ^ (h1 | h2));            // sparse and no exception hit
+    uint32_t e3 = cls2 + (lo & 0xFFFFu) * st.c_row_bytes;   // dense entry (fd, cls)
+    asm("{\n\t.reg .pred p;\n\t.reg .u32 a;\n\tsetp.ne.u32 p, %1, 0;\n\tadd.u32 a, %0, %2;\n\t@p ld.shared.u16 %0, [a];\n\t}"
         : "+r"(e3)
-        : "r"(need));
+        : "r"(need), "r"(base));
     const uint32_t ex = __byte_perm(hi, 0, h1 ? 0x4410 : 0x4432);
     return sp ? (need ? e3 : ex) : lo;
 }

@@ -155,6 +155,8 @@ def _decode_compact(t):
     rec = blob[d["compact_sparse_off"]:d["compact_sparse_off"] + (S - nd) * 8].view(np.uint32).reshape(-1, 2)
     fd = rec[:, 0] & 0xFFFF
     c1, c2 = (rec[:, 0] >> 16) & 0xFF, rec[:, 0] >> 24
+    assert ((c1 == 0xFF) | (c1 % 2 == 0)).all() and ((c2 == 0xFF) | (c2 % 2 == 0)).all()
+    c1, c2 = np.where(c1 == 0xFF, 0xFF, c1 // 2), np.where(c2 == 0xFF, 0xFF, c2 // 2)  # doubled classes
     t1, t2 = rec[:, 1] & 0xFFFF, rec[:, 1] >> 16
     cls = np.arange(C)[None, :]
     sparse = np.where(cls == c1[:, None], t1[:, None],
@@ -256,3 +258,13 @@ def test_no_device_fails_loudly():
     with pytest.raises(ac.AcError) as e:
         ac.build([b"he"], device=0)
     assert e.value.status in (ac.AC_ERR_NO_DEVICE, ac.AC_ERR_CUDA)
+
+
+def test_compact_rejects_wide_alphabets():
+    """COMPACT stores doubled classes in bytes: at most 127 classes."""
+    ok = [bytes([b]) + bytes([b + 1]) for b in range(0, 120, 2)]  # 121 classes
+    t = ac.compile_table(ok, compact=True)
+    assert t.info["n_classes"] <= 127 and t.info["compact_bytes"] > 0
+    wide = [bytes([b, (b * 7) % 256]) for b in range(200)]
+    with pytest.raises(ac.AcError):
+        ac.compile_table(wide, compact=True)
