@@ -120,8 +120,9 @@ typedef struct {
     /* COMPACT encoding (valid when compact_bytes != 0): byte layout
      * [dense rows: compact_dense x compact_dstride u16]
      * [sparse records at compact_sparse_off: (n_states - compact_dense) x 8 B,
-     *  lo32 = fd | 2 c1 << 16 | 2 c2 << 24 (doubled classes, 0xFF = none),
-     *  hi32 = t1 | t2 << 16]
+     *  lo32 = 2 c1 | 2 c2 << 8 | fd << 16 (doubled classes, 0xFF = none),
+     *  hi32 = t1 | t2 << 16]; every entry (dense row cell, t1, t2) is
+     *  2 x + flag, x = compact id of the next state, flag = output(x) != {}
      * [output table at compact_out_off: (compact_od + compact_os) x
      *  (u32 payload, u32 count)], compact ids: 0 = root, then other dense
      * states, dense output states, sparse output states, other sparse: the

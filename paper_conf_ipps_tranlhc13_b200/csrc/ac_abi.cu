@@ -159,6 +159,12 @@ static SttView view_of(const ac_stt *h, int v) {
     s.c_row_bytes = 2 * h->host.c_dstride;
     s.c_sparse_x0 = h->host.c_sparse_off - 8u * h->host.c_dense;
     s.c_out_x0 = h->host.c_out_off - 8u * (h->host.c_dense - h->host.c_od);
+    s.c_rec_bytes = 8;
+    s.c_two = 2;
+    s.c_mtwo = 0xFFFFFFFEu;
+    s.c_half = 0x80000000u;
+    s.c_k16 = 0x10000u;
+    s.c_rep = 0x0101u;
     s.stt2 = v ? h->d_stt2 : nullptr;  // only the staged kernel walks two bytes per lookup
     s.stride2 = h->host.stride2;
     s.n_classes = h->host.n_classes;

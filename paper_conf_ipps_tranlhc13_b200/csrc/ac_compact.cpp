@@ -20,8 +20,8 @@
 //     is one subtraction: oidx = x - (c_dense - c_od); each table slot holds
 //     (payload, count) exactly like the dense rows' output summary.
 //
-// Entries keep the dense layout's convention: bit 15 = output(next) != {},
-// bits 0..14 = next state (COMPACT requires <= 32768 states and C <= 127).
+// Entries are 2 x + flag: x = the next state's compact id, flag =
+// output(next) != {} (COMPACT requires <= 32768 states and C <= 127).
 // The device class map of a COMPACT automaton holds 2 x class: the byte
 // offset of the class's column inside a dense row, compared directly with
 // the records' (doubled) exception classes.
@@ -103,7 +103,8 @@ bool compact_table(ac_table &t, size_t budget) {
         if (!dense[s] && !is_out(s)) perm.push_back(s);
     std::vector<uint32_t> inv(S);
     for (uint32_t x = 0; x < S; x++) inv[perm[x]] = x;
-    auto enc = [&](uint16_t e) -> uint16_t { return (uint16_t)(inv[e & 0x7fffu] | (e & 0x8000u)); };
+    // COMPACT entry = 2 x + flag (x = compact id of the next state)
+    auto enc = [&](uint16_t e) -> uint16_t { return (uint16_t)((inv[e & 0x7fffu] << 1) | (e >> 15)); };
 
     uint32_t words = (C + 1) / 2;
     if (words % 2 == 0) words++;
@@ -117,9 +118,10 @@ bool compact_table(ac_table &t, size_t budget) {
             std::memcpy(&blob[((size_t)x * dstride + c) * 2], &e, 2);
         }
     }
-    // sparse records: lo = fd | 2 c1 << 16 | 2 c2 << 24, hi = t1 | t2 << 16
+    // sparse records: lo = 2 c1 | 2 c2 << 8 | fd << 16, hi = t1 | t2 << 16
     // (classes doubled, as in the COMPACT class map: a doubled class is the
-    // byte offset of its column in a dense row; 0xFF = no exception)
+    // byte offset of its column in a dense row; 0xFF = no exception; fd is a
+    // plain compact id, t1 and t2 are entries)
     std::vector<uint32_t> fd(S, 0);
     for (uint32_t s = 1; s < S; s++)
         if (!dense[s]) fd[s] = dense[t.fail[s]] ? t.fail[s] : fd[t.fail[s]];
@@ -136,7 +138,7 @@ bool compact_table(ac_table &t, size_t budget) {
                 k++;
             }
         }
-        const uint32_t lo = inv[fd[s]] | (cls[0] << 16) | (cls[1] << 24);
+        const uint32_t lo = cls[0] | (cls[1] << 8) | (inv[fd[s]] << 16);
         const uint32_t hi = (uint32_t)tgt[0] | ((uint32_t)tgt[1] << 16);
         uint8_t *r = &blob[dense_bytes + (size_t)(x - nd) * 8];
         std::memcpy(r, &lo, 4);

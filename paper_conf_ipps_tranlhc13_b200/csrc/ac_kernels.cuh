@@ -101,36 +101,58 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
     }
 }
 
-// The entry delta(s, cls): next state in the low bits, output flag on top.
+// The entry delta(s, cls).  Dense tiers: next state in the low bits, output
+// flag on top.  COMPACT: e = 2 x + flag (x = next state, compact id).
 // COMPACT: a dense row, or a sparse record's exception, or the dense row of
 // the record's default state fd(s) -- at most two shared-memory loads, issued
 // as predicated loads so lanes in dense and sparse states never diverge.
 // (Each predicated load's destination register is pre-loaded with a value
 // that is dead afterwards -- its own address -- so no zeroing moves are
 // needed; write-only "=r" outputs made ptxas spill 372 B per thread.)
+// The COMPACT walk is bound by the ALU pipe (ncu: 86-89 % busy, FMA pipe
+// 14 %), so its shifts, masks and field extractions are written as
+// multiply-adds and multiply-highs by RUN-TIME constants (SttView c_*), which
+// the compiler can neither strength-reduce back to shifts nor fold: they
+// issue on the otherwise idle FMA pipe.
 __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls2) {
     // cls2 = 2 x class (the COMPACT class map is pre-doubled): the byte
     // offset of column cls inside a dense row, and the form in which the
     // sparse records store their exception classes
     const uint32_t sp = s >= st.c_dense;
-    uint32_t lo, hi = cls2 + s * st.c_row_bytes;  // dense entry (s, cls) (garbage if sparse)
-    asm("mad.lo.u32 %0, %1, 8, %2;" : "=r"(lo) : "r"(s), "r"(base + st.c_sparse_x0));  // sparse record of s
+    uint32_t hi = cls2 + s * st.c_row_bytes;                   // dense entry (s, cls) (garbage if sparse)
+    uint32_t lo = s * st.c_rec_bytes + (base + st.c_sparse_x0);  // sparse record of s (garbage if dense)
     asm("{\n\t.reg .pred p;\n\t.reg .u32 a;\n\tsetp.ne.u32 p, %2, 0;\n\t"
         "add.u32 a, %1, %3;\n\t"
         "@p ld.shared.v2.u32 {%0, %1}, [%0];\n\t"
         "@!p ld.shared.u16 %0, [a];\n\t}"
         : "+r"(lo), "+r"(hi)
         : "r"(sp), "r"(base));
-    // sparse: lo = fd | c1 << 16 | c2 << 24 (exception classes doubled), hi = t1 | t2 << 16
-    const uint32_t x = lo ^ __byte_perm(cls2, 0, 0x0000);  // byte k of x is 0 iff byte k of lo == cls2
-    const uint32_t h1 = (x & 0x00FF0000u) == 0, h2 = (x & 0xFF000000u) == 0;
-    const uint32_t need = sp & (1u ^ (h1 | h2));            // sparse and no exception hit
-    uint32_t e3 = cls2 + (lo & 0xFFFFu) * st.c_row_bytes;   // dense entry (fd, cls)
+    // sparse: lo = c1 | c2 << 8 | fd << 16 (exception classes doubled), hi = t1 | t2 << 16
+    const uint32_t rep = cls2 * st.c_rep;                      // cls2 in bytes 0 and 1
+    const uint32_t h1 = ((lo ^ rep) & 0xFFu) == 0, h2 = ((lo ^ rep) & 0xFF00u) == 0;
+    const uint32_t need = sp & (1u ^ (h1 | h2));                // sparse and no exception hit
+    uint32_t e3 = cls2 + __umulhi(lo, st.c_k16) * st.c_row_bytes;  // dense entry (fd, cls)
     asm("{\n\t.reg .pred p;\n\t.reg .u32 a;\n\tsetp.ne.u32 p, %1, 0;\n\tadd.u32 a, %0, %2;\n\t@p ld.shared.u16 %0, [a];\n\t}"
         : "+r"(e3)
         : "r"(need), "r"(base));
     const uint32_t ex = __byte_perm(hi, 0, h1 ? 0x4410 : 0x4432);
     return sp ? (need ? e3 : ex) : lo;
+}
+
+// Entry -> next state and output flag.
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t state_of(uint32_t e, const SttView &st) {
+    if constexpr (TIER == AC_TIER_COMPACT)
+        return __umulhi(e, st.c_half);  // e >> 1 on the FMA pipe
+    else
+        return e & EntryBits<E>::MASK;
+}
+template <typename E, int TIER>
+__device__ __forceinline__ uint32_t flag_of(uint32_t e, uint32_t x, const SttView &st) {
+    if constexpr (TIER == AC_TIER_COMPACT)
+        return e + x * st.c_mtwo;  // e - 2 x (IMAD)
+    else
+        return e >> (8 * sizeof(E) - 1);
 }
 
 template <typename E, int TIER>
@@ -146,7 +168,7 @@ __device__ __forceinline__ uint32_t next_entry(const E *s_stt, const SttView &st
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uint8_t *s_cmap, const E *s_stt,
                                             const SttView &st) {
-    return next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]) & EntryBits<E>::MASK;
+    return state_of<E, TIER>(next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]), st);
 }
 
 // COMPACT output table slot of output state s: (payload, count).
@@ -304,7 +326,8 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
                                         bool live, const uint8_t *s_cmap, const E *s_stt, const SttView &st,
                                         const ScanOut &so) {
     const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
-    s = e & EntryBits<E>::MASK;
+    s = state_of<E, TIER>(e, st);
+    const uint32_t flag = flag_of<E, TIER>(e, s, st);
     // Predication pays where matches are dense (C2-like dictionaries, which are
     // what land in COMPACT); with rare flags (C1/C3/C4) the predicated loads
     // and store cost issue slots on every byte (measured: C1 list 2.6x slower),
@@ -314,7 +337,7 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
         // Branch-free for the common cases: predicated loads of the output
         // summary and a predicated store of a single-output match; only
         // multi-output states (and saturated counts) take a branch.
-        const uint32_t f = ((e & EntryBits<E>::FLAG) != 0) & (live ? 1u : 0u);
+        const uint32_t f = flag & (live ? 1u : 0u);
         const uint2 o = out_info_pred<E, TIER, MODE == MODE_EMIT_OPT>(s_stt, st, s, f);
         uint32_t c = o.y;
         if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
@@ -339,7 +362,7 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
         }
         return;
     }
-    if ((e & EntryBits<E>::FLAG) && live) emit_outputs<E, TIER, MODE>(s, key0, cnt, wp, s_stt, st, so);
+    if (flag && live) emit_outputs<E, TIER, MODE>(s, key0, cnt, wp, s_stt, st, so);
 }
 
 // NEXT-4: one lookup for two bytes.  T2[s][c1*C + c2] =
@@ -357,7 +380,7 @@ __device__ __forceinline__ void ac_step2(uint32_t &s, uint32_t &cnt, uint64_t &w
     const uint32_t e = __ldg(st.stt2 + s * st.stride2 + c1 * st.n_classes + c2);
     if ((e & (T2_FIN | T2_MID)) && live) {
         if (e & T2_MID) {
-            const uint32_t mid = next_entry<E, TIER>(s_stt, st, s, c1) & EntryBits<E>::MASK;
+            const uint32_t mid = state_of<E, TIER>(next_entry<E, TIER>(s_stt, st, s, c1), st);
             emit_outputs<E, TIER, MODE>(mid, key1, cnt, wp, s_stt, st, so);
         }
         if (e & T2_FIN) emit_outputs<E, TIER, MODE>(e & T2_MASK, key2, cnt, wp, s_stt, st, so);
@@ -739,12 +762,22 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
                     for (int bb = 15; bb >= 0; --bb) {
                         const uint32_t e = next_entry<E, TIER>(s_stt, st, st0, s_cmap[byte_of(v[0], bb)]);
-                        st0 = e & EntryBits<E>::MASK;
-                        fm = (fm << 1) | (e >> 15);  // byte bb's flag ends at bit bb
-                        if (bb & 1)
-                            odd = st0;
-                        else
-                            hist[bb >> 1] = __byte_perm(odd, st0, 0x5410);  // (odd, even << 16)
+                        st0 = state_of<E, TIER>(e, st);
+                        const uint32_t f = flag_of<E, TIER>(e, st0, st);
+                        // byte bb's flag ends at bit bb; hist[i] = (state at 2i+1, state at 2i << 16)
+                        if constexpr (TIER == AC_TIER_COMPACT) {
+                            fm = fm * st.c_two + f;  // FMA pipe
+                            if (bb & 1)
+                                odd = st0;
+                            else
+                                hist[bb >> 1] = odd + st0 * st.c_k16;
+                        } else {
+                            fm = (fm << 1) | f;
+                            if (bb & 1)
+                                odd = st0;
+                            else
+                                hist[bb >> 1] = __byte_perm(odd, st0, 0x5410);
+                        }
                     }
                     s[0] = st0;
                     if (!live[0]) fm = 0;
@@ -754,29 +787,34 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                         const uint64_t *const last = reinterpret_cast<const uint64_t *>(wp[0]);
                         int32_t nk = -(int32_t)cnt[0];
                         const int32_t nq = -(int32_t)so.q;
-                        while (__any_sync(0xffffffffu, fm)) {
-                            if (fm) {
-                                const int bb = 31 - __clz(fm);
-                                fm ^= 1u << bb;
-                                const int i = bb >> 1;
-                                const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
-                                const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
-                                const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
-                                const uint32_t pr = (i & 4) ? b1 : b0;
-                                const uint32_t x = __byte_perm(pr, 0, (bb & 1) ? 0x4410 : 0x4432);
-                                const uint2 o = compact_or_row_out<E, TIER>(s_stt, st, x);
-                                // key = (start << 24) | pid, start = chunk start + bb (pid < 2^24)
-                                const uint32_t kl = (uint32_t)bb << 24;
-                                if (o.y == 1) {
-                                    st_global_if(last, nk, kb[0] + (kl | o.x), nk > nq);
-                                    --nk;
-                                } else {
-                                    for (uint32_t j = o.x + o.y; j > o.x; --j) {
-                                        st_global_if(last, nk, kb[0] + (kl | __ldg(st.out_ids + j - 1)), nk > nq);
-                                        --nk;
-                                    }
-                                }
+                        // A warp-uniform trip count (the most flags any lane
+                        // holds) instead of a divergent while-any loop: no
+                        // reconvergence bookkeeping, predicated body.
+                        const uint32_t iters = __reduce_max_sync(0xffffffffu, (uint32_t)__popc(fm));
+                        for (uint32_t it = 0; it < iters; ++it) {
+                            uint32_t bb;  // highest flagged byte left (0xffffffff if none)
+                            asm("bfind.u32 %0, %1;" : "=r"(bb) : "r"(fm));
+                            const uint32_t act = fm != 0;
+                            fm &= ~(1u << (bb & 31u));
+                            const uint32_t i = bb >> 1;
+                            const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
+                            const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
+                            const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
+                            const uint32_t pr = (i & 4) ? b1 : b0;
+                            const uint32_t x = __byte_perm(pr, 0, (bb & 1) ? 0x4410 : 0x4432);
+                            const uint2 o = out_info_pred<E, TIER, true>(s_stt, st, x, act);
+                            uint32_t c = o.y;
+                            if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
+                                c = __ldg(st.out_off + x + 1) - __ldg(st.out_off + x);
+                            // key = (start << 24) | pid, start = chunk start + bb (pid < 2^24)
+                            const uint64_t k0 = kb[0] + ((uint64_t)(bb & 15u) << 24);
+                            st_global_if(last, nk, k0 + o.x, (c == 1u) & (nk > nq));
+                            if (__any_sync(0xffffffffu, c > 1u)) {  // multi-output states (rare)
+                                for (uint32_t j = 0; j < c && c > 1u; ++j)
+                                    st_global_if(last, nk - (int32_t)j, k0 + __ldg(st.out_ids + o.x + c - 1 - j),
+                                                 nk - (int32_t)j > nq);
                             }
+                            nk -= (int32_t)c;
                         }
                         cnt[0] = (uint32_t)(-nk);
                     } else

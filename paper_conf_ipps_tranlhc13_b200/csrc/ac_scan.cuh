@@ -34,6 +34,9 @@ struct SttView {
     // c_sparse_x0 + 8 x, output slot of output state x at c_out_x0 + 8 x
     // (both x0 wrap around modulo 2^32 on purpose)
     uint32_t c_dense, c_row_bytes, c_sparse_x0, c_out_x0;
+    // run-time constants of the COMPACT walk (see compact_next): 8, 2, -2,
+    // 2^31, 2^16, 0x0101 -- multiplied, never shifted, to load the FMA pipe
+    uint32_t c_rec_bytes, c_two, c_mtwo, c_half, c_k16, c_rep;
     // two-byte table (NEXT-4): row s, column c1 * n_classes + c2; NULL = off
     const uint32_t *stt2;
     uint32_t stride2, n_classes;

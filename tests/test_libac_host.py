@@ -153,8 +153,8 @@ def _decode_compact(t):
     blob = t.compact
     dense = blob[:nd * ds * 2].view(np.uint16).reshape(nd, ds)[:, :C].astype(np.int64)
     rec = blob[d["compact_sparse_off"]:d["compact_sparse_off"] + (S - nd) * 8].view(np.uint32).reshape(-1, 2)
-    fd = rec[:, 0] & 0xFFFF
-    c1, c2 = (rec[:, 0] >> 16) & 0xFF, rec[:, 0] >> 24
+    fd = rec[:, 0] >> 16
+    c1, c2 = rec[:, 0] & 0xFF, (rec[:, 0] >> 8) & 0xFF
     assert ((c1 == 0xFF) | (c1 % 2 == 0)).all() and ((c2 == 0xFF) | (c2 % 2 == 0)).all()
     c1, c2 = np.where(c1 == 0xFF, 0xFF, c1 // 2), np.where(c2 == 0xFF, 0xFF, c2 // 2)  # doubled classes
     t1, t2 = rec[:, 1] & 0xFFFF, rec[:, 1] >> 16
@@ -162,6 +162,7 @@ def _decode_compact(t):
     sparse = np.where(cls == c1[:, None], t1[:, None],
                       np.where(cls == c2[:, None], t2[:, None], dense[fd]))
     E = np.concatenate([dense, sparse.astype(np.int64)])
+    E = (E >> 1) | ((E & 1) << 15)  # entries are 2 x + flag -> x | flag << 15
     nout = d["compact_od"] + d["compact_os"]
     ot = blob[d["compact_out_off"]:d["compact_out_off"] + nout * 8].view(np.uint32).reshape(-1, 2)
     return E, ot
