@@ -586,11 +586,19 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
             : "memory");
     } while (!done);
 }
-__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y, uint64_t *bar) {
+// The text is streamed exactly once: its TMA loads carry an L2 evict-first
+// policy so they do not push the automaton (L1/L2-resident tiers) out of L2.
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y, uint64_t *bar,
+                                            uint64_t policy) {
     asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], "
-        "[%4];" ::"r"(smem_u32(dst)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint "
+        "[%0], [%1, {%2, %3}], [%4], %5;" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar)), "l"(policy)
         : "memory");
 }
 
@@ -644,6 +652,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     const bool tma_halo = (uint64_t)nh0 * W <= L;  // the halo window lies inside the next chain
     const uint32_t nh = tma_halo ? nh0 : 0;
     const uint32_t m = nh + (uint32_t)(L / W);
+    const uint64_t pol = l2_evict_first_policy();
 
     auto issue = [&](uint32_t j) {
         const uint32_t slot = j % NST;
@@ -656,7 +665,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
             y = (int)row0;
         }
         mbar_expect_tx(&wbar[slot], Sh::SLOT);
-        tma_load_2d(wring + slot * Sh::SLOT, &tmap, x, y, &wbar[slot]);
+        tma_load_2d(wring + slot * Sh::SLOT, &tmap, x, y, &wbar[slot], pol);
     };
     if (lane == 0)
         for (uint32_t j = 0; j < (uint32_t)NST && j < m; j++) issue(j);
