@@ -271,8 +271,10 @@ def run_ours(args):
     for nm, t in zip(names, kms):
         if "scan" in nm:
             byts = n + (out_bytes if "emit" in nm else 0)
+        elif "gather" in nm:
+            byts = 2 * out_bytes  # every record read from its scratch slot and written once
         else:
-            byts = 16 * (n // 1024)
+            byts = 0  # offset scan / overflow re-walk: latency-bound bookkeeping
         kern.append({"name": nm, "ms": float(t), "share": float(t / ms), "alg_bytes": int(byts)})
     dom = max(kern, key=lambda k: k["ms"])
     hbm, hbm_src, pk = peaks()

@@ -38,6 +38,8 @@ def main():
     p.add_argument("--variants", default="1,2,3,4,5,6,7")
     p.add_argument("--tiers", default="auto")
     p.add_argument("--global-kernel", action="store_true")
+    p.add_argument("--two-pass", default="0", help="list-mode placements to time: 0 single pass (block gather), "
+                   "1 count+emit passes, 2 single pass via offset scan + k_gather")
     a = p.parse_args()
     w = synth.make(a.config, n=a.n or None)
     n = w.text.size
@@ -49,12 +51,12 @@ def main():
         stt = ac.build(w.patterns, tier=tiers[tname])
         cnt = ac.count(stt, text)
         out = torch.empty(max(1, cnt), dtype=torch.int64, device="cuda")
-        settings = [(ac.KERNEL_STAGED, int(v)) for v in a.variants.split(",")]
+        settings = [(ac.KERNEL_STAGED, int(v), int(tp)) for v in a.variants.split(",") for tp in a.two_pass.split(",")]
         if a.global_kernel:
-            settings.append((ac.KERNEL_GLOBAL, 0))
+            settings.append((ac.KERNEL_GLOBAL, 0, 0))
         ref = None
-        for kernel, v in settings:
-            knobs = dict(kernel=kernel, variant=v)
+        for kernel, v, tp in settings:
+            knobs = dict(kernel=kernel, variant=v, two_pass=tp)
             try:
                 ac.match_async(stt, text, None, res, **knobs)
             except ac.AcError as e:
@@ -67,7 +69,7 @@ def main():
             h = int(torch.sum(out[:cnt] * 0x9E3779B1 % 1000003).item())
             ref = h if ref is None else ref
             print(json.dumps({"config": a.config, "n": n, "tier": stt.tier_name, "hot_rows": stt.info["hot_rows"],
-                              "kernel": kernel, "variant": v, "count_ms": round(t_count, 4),
+                              "kernel": kernel, "variant": v, "two_pass": tp, "count_ms": round(t_count, 4),
                               "list_ms": round(t_list, 4), "count_gbps": round(n * 8 / t_count / 1e6, 1),
                               "list_gbps": round(n * 8 / t_list / 1e6, 1), "matches": cnt,
                               "same_list": h == ref}), flush=True)
