@@ -159,8 +159,12 @@ typedef struct {
                               scratch slot during the single emitting pass
                               (0 = auto from cap); chains with more are
                               re-scanned straight into place                 */
-    uint32_t two_pass;     /* list mode: 1 = count pass + emit pass instead
-                              of the single pass (ablation / fallback)       */
+    uint32_t two_pass;     /* list mode: 0 = single emitting pass (chain
+                              offsets computed inside the staged scan when
+                              the text pointer is 16-byte aligned, else by
+                              a separate offset scan); 1 = count pass + emit
+                              pass (ablation / fallback); 2 = single pass
+                              with the separate offset scan (ablation)     */
     uint32_t stride;       /* 0 = the table's default, 1 = force one byte
                               per lookup even if a two-byte table exists     */
     uint32_t n_events;     /* pairs available in `events`                    */

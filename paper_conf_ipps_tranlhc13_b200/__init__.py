@@ -202,7 +202,7 @@ def _check_text(text: torch.Tensor):
 def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, scratch_slots: int = 0,
            two_pass: bool = False, events=None, stride: int = 0):
     o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, scratch_slots,
-                      1 if two_pass else 0, stride, 0, None)
+                      int(two_pass), stride, 0, None)
     if events:
         arr = (ctypes.c_void_p * (2 * len(events)))(*[e.cuda_event for pair in events for e in pair])
         o.n_events = len(events)

@@ -373,9 +373,16 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         return scan(MODE_COUNT_TOTAL, "k_scan_global(count)", "k_scan_staged(count)");
     }
     // --- list mode workspace: counts | chain_end | list | tile_state | counters
-    const bool two_pass = opts && opts->two_pass;
+    const bool two_pass = opts && opts->two_pass == 1;
+    // in-kernel offsets: the staged kernel places its chains (decoupled
+    // look-back per CTA) when the main region starts the list and the tail
+    // is short; k_gather places the tail.  two_pass = 2 forces k_offsets.
+    const bool place = !two_pass && !(opts && opts->two_pass == 2) && g.n_chains > 0 && ra.n_chains == 0 &&
+                       rb.n_chains <= 256;
+    const uint64_t R = (uint64_t)cfg.warps * 32 * cfg.k;
+    const uint64_t n_lb = place ? (g.n_chains + R - 1) / R : 0;  // staged CTAs
     const size_t tiles = offsets_tiles(n_chains);
-    const size_t bytes = n_chains * 8 * 3 + tiles * 8 + 16;
+    const size_t bytes = n_chains * 8 * 3 + tiles * 8 + 16 + n_lb * 8;
     void *ws = nullptr;
     AC_CUDA(cudaMallocAsync(&ws, bytes, stream), "cudaMallocAsync(workspace)");
     uint64_t *counts = static_cast<uint64_t *>(ws);
@@ -384,6 +391,10 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     uint64_t *tile_state = list + n_chains;
     unsigned int *counter = reinterpret_cast<unsigned int *>(tile_state + tiles);
     unsigned int *list_n = counter + 1;
+    unsigned long long *lb = place ? reinterpret_cast<unsigned long long *>(counter + 4) : nullptr;
+    so.tile_state = lb;
+    so.chain_end_w = chain_end;
+    TailPlace tp{lb, n_lb, rb.chain0, rb.n_chains, cap};
     so.chain_counts = counts;
     so.chain_end = chain_end;
     // single pass: each chain keeps its first q records in a scratch slot
@@ -403,7 +414,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         so.q = (uint32_t)q;
     }
     auto run = [&]() -> ac_status {
-        AC_CUDA(cudaMemsetAsync(tile_state, 0, tiles * 8 + 16, stream), "memset workspace");
+        AC_CUDA(cudaMemsetAsync(tile_state, 0, tiles * 8 + 16 + n_lb * 8, stream), "memset workspace");
         if (two_pass) {
             ac_status rc = scan(MODE_COUNT_CHAINS, "k_scan_global(count)", "k_scan_staged(count)");
             if (rc != AC_OK) return rc;
@@ -415,12 +426,15 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         }
         ac_status rc = scan(MODE_EMIT_OPT, "k_scan_global(emit1)", "k_scan_staged(emit1)");
         if (rc != AC_OK) return rc;
+        if (!place) {
+            pre();
+            AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream),
+                    "k_offsets");
+            post("k_offsets");
+        }
         pre();
-        AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream), "k_offsets");
-        post("k_offsets");
-        pre();
-        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, h->num_sms,
-                              stream),
+        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, tp,
+                              h->num_sms, stream),
                 "k_gather");
         post("k_gather");
         pre();

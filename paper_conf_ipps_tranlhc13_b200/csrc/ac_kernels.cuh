@@ -602,6 +602,85 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
         : "memory");
 }
 
+// ------------------------------------------------- in-kernel offsets (a9)
+// Epilogue of the single emitting pass when the main region starts the list
+// (no head chains): a CTA's chains are consecutive in canonical order, so
+// the CTA needs only the match total of the CTAs before it -- a decoupled
+// look-back over one word per CTA (CTAs are dispatched in index order, so
+// every predecessor is running or done; warp 0 reads 32 predecessors per
+// step) -- to write every chain's end offset.  This replaces the k_offsets
+// launch.  Shared memory for the exchange is the warps' own (finished) TMA
+// ring slots.
+__device__ __forceinline__ uint64_t ld_acquire_u64(const unsigned long long *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u64(unsigned long long *p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+template <int K>
+__device__ __forceinline__ void place_chains(const ScanOut &so, const StagedGeom &g, uint8_t *wring, uint8_t *ring,
+                                             int warp_ring, int warps, uint64_t row0, const uint32_t (&cnt)[K],
+                                             const bool (&live)[K]) {
+    const int lane = threadIdx.x & 31;
+    // warp-level inclusive scan in canonical chain order (k major, lane minor)
+    uint64_t incl[K];
+    uint64_t run = 0;
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        uint64_t v = live[k] ? cnt[k] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint64_t y = __shfl_up_sync(0xffffffffu, v, o);
+            if (lane >= o) v += y;
+        }
+        incl[k] = run + v;
+        run += __shfl_sync(0xffffffffu, v, 31);
+    }
+    uint64_t *wslot = reinterpret_cast<uint64_t *>(wring);
+    __syncwarp();
+    if (lane == 0) wslot[0] = run;  // this warp's total
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        uint64_t tot = 0;
+        for (int w = 0; w < warps; w++) tot += reinterpret_cast<uint64_t *>(ring + w * warp_ring)[0];
+        uint64_t prefix = 0;
+        if (blockIdx.x == 0) {
+            if (lane == 0) st_release_u64(&so.tile_state[0], LB_INC | tot);
+        } else {
+            if (lane == 0) st_release_u64(&so.tile_state[blockIdx.x], LB_AGG | tot);
+            int64_t p = (int64_t)blockIdx.x - 1;  // nearest predecessor of the window
+            while (true) {
+                const int64_t idx = p - lane;
+                uint64_t st = idx >= 0 ? ld_acquire_u64(&so.tile_state[idx]) : LB_INC;  // before CTA 0: 0
+                while (__any_sync(0xffffffffu, (st >> 62) == 0))
+                    if ((st >> 62) == 0) st = ld_acquire_u64(&so.tile_state[idx]);  // not yet published
+                const uint32_t inc = __ballot_sync(0xffffffffu, (st & LB_INC) == LB_INC);
+                const int stop = inc ? __ffs(inc) - 1 : 31;  // lanes 0..stop contribute
+                uint64_t val = lane <= stop ? (st & LB_VAL) : 0;
+                for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(0xffffffffu, val, o);
+                prefix += val;
+                if (inc) break;
+                p -= 32;
+            }
+            if (lane == 0) st_release_u64(&so.tile_state[blockIdx.x], LB_INC | (prefix + tot));
+        }
+        if (lane == 0)  // exclusive prefix of every warp, into its slot (word 1)
+            for (int w = 0; w < warps; w++) {
+                uint64_t *ws = reinterpret_cast<uint64_t *>(ring + w * warp_ring);
+                ws[1] = prefix;
+                prefix += ws[0];
+            }
+    }
+    __syncthreads();
+    const uint64_t wpre = wslot[1];
+#pragma unroll
+    for (int k = 0; k < K; k++)
+        if (live[k]) so.chain_end_w[g.chain0 + row0 + k * 32 + lane] = wpre + incl[k];
+}
+
 // ------------------------------------------- k_scan_staged (warp-private TMA)
 template <int WARPS, int K, int W, int NST, int SWIZZLE>
 struct StagedShape {
@@ -642,7 +721,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
         if (so.res->status != AC_OK) return;  // capacity exceeded: write nothing
     }
     const uint64_t row0 = (uint64_t)blockIdx.x * (WARPS * Sh::ROWS) + (uint64_t)warp * Sh::ROWS;
-    if (row0 >= g.n_chains) return;  // idle warp (no later CTA barrier)
+    // in-kernel placement ends with CTA barriers: idle warps stay (no tiles)
+    const bool place = MODE == MODE_EMIT_OPT && so.tile_state != nullptr;
+    const bool idle = row0 >= g.n_chains;
+    if (idle && !place) return;  // idle warp (no later CTA barrier)
 
     uint8_t *wring = ring + warp * Sh::WARP_RING;
     uint64_t *wbar = bars + warp * NST;
@@ -651,7 +733,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     const uint32_t nh0 = (H + W - 1) / W;
     const bool tma_halo = (uint64_t)nh0 * W <= L;  // the halo window lies inside the next chain
     const uint32_t nh = tma_halo ? nh0 : 0;
-    const uint32_t m = nh + (uint32_t)(L / W);
+    const uint32_t m = idle ? 0u : nh + (uint32_t)(L / W);
     const uint64_t pol = l2_evict_first_policy();
 
     auto issue = [&](uint32_t j) {
@@ -887,6 +969,9 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
         for (int k = 0; k < K; k++)
             if (live[k]) so.chain_counts[g.chain0 + row0 + k * 32 + lane] = cnt[k];
+    }
+    if constexpr (MODE == MODE_EMIT_OPT) {
+        if (place) place_chains<K>(so, g, wring, ring, Sh::WARP_RING, WARPS, row0, cnt, live);
     }
 
     if constexpr (MODE == MODE_COUNT_TOTAL) {

@@ -123,24 +123,57 @@ size_t offsets_tiles(uint64_t n) { return (size_t)((n + OTILE - 1) / OTILE); }
 // ------------------------------------------------------------- k_gather
 // One warp per chain (grid-stride): a chain whose count fits its scratch slot
 // is copied, coalesced, from the tail of the slot to [chain_end - cnt,
-// chain_end); an overflowed chain is appended to the re-walk list.
-__global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ counts,
-                                                const uint64_t *__restrict__ chain_end, uint64_t n_chains,
-                                                const uint64_t *__restrict__ scratch, uint32_t q,
-                                                uint64_t *__restrict__ out, const ac_result *res, uint64_t *list,
-                                                unsigned int *list_n) {
-    if (res->status != AC_OK) return;
+// chain_end); an overflowed chain is appended to the re-walk list.  With a
+// TailPlace (the staged kernel already placed the main chains) every CTA
+// also derives the grand total and the tail chains' offsets itself and CTA 0
+// writes the count and the capacity status.
+static constexpr uint64_t kMaxTail = 256;
+
+__global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ counts, uint64_t *chain_end,
+                                                uint64_t n_chains, const uint64_t *__restrict__ scratch, uint32_t q,
+                                                uint64_t *__restrict__ out, ac_result *res, uint64_t *list,
+                                                unsigned int *list_n, TailPlace tp) {
     const int lane = threadIdx.x & 31;
+    uint64_t main_total = 0;
+    if (tp.tile_state) {
+        __shared__ unsigned long long s_tail[256 / 32];
+        main_total = tp.tile_state[tp.n_tiles - 1] & LB_VAL;
+        unsigned long long t = threadIdx.x < tp.tail_n ? counts[tp.tail_c0 + threadIdx.x] : 0;
+        for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+        if (lane == 0) s_tail[threadIdx.x >> 5] = t;
+        __syncthreads();
+        uint64_t total = main_total;
+        for (int i = 0; i < 256 / 32; i++) total += s_tail[i];
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            res->count = total;
+            res->status = total > tp.cap ? (uint32_t)AC_ERR_CAPACITY : (uint32_t)AC_OK;
+        }
+        if (total > tp.cap) return;  // capacity exceeded: write nothing
+    } else if (res->status != AC_OK) {
+        return;
+    }
     const uint64_t warps = (uint64_t)gridDim.x * (blockDim.x >> 5);
     for (uint64_t c = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < n_chains; c += warps) {
         const uint64_t cnt = counts[c];
+        uint64_t end;
+        if (tp.tile_state && c >= tp.tail_c0) {
+            // tail chain: main total + inclusive sum of the tail counts up to c
+            unsigned long long v = 0;
+            for (uint64_t j = tp.tail_c0 + lane; j <= c; j += 32) v += counts[j];
+            for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+            end = main_total + v;
+            if (lane == 0) chain_end[c] = end;  // k_rewalk reads it for listed chains
+        } else {
+            if (cnt == 0) continue;
+            end = chain_end[c];
+        }
         if (cnt == 0) continue;
         if (cnt > q) {
             if (lane == 0) list[atomicAdd(list_n, 1u)] = c;
             continue;
         }
         const uint64_t *src = scratch + c * q + (q - cnt);
-        uint64_t *dst = out + chain_end[c] - cnt;
+        uint64_t *dst = out + end - cnt;
         // four records in flight per lane before the stores
         uint64_t i = lane;
         for (; i + 96 < cnt; i += 128) {
@@ -155,13 +188,15 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
     }
 }
 
-cudaError_t launch_gather(const uint64_t *counts, const uint64_t *chain_end, uint64_t n_chains,
-                          const uint64_t *scratch, uint32_t q, uint64_t *out, const ac_result *res, uint64_t *list,
-                          unsigned int *list_n, int num_sms, cudaStream_t stream) {
+cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t n_chains,
+                          const uint64_t *scratch, uint32_t q, uint64_t *out, ac_result *res,
+                          uint64_t *list, unsigned int *list_n, const TailPlace &tp, int num_sms,
+                          cudaStream_t stream) {
     if (n_chains == 0) return cudaSuccess;
+    if (tp.tile_state && tp.tail_n > kMaxTail) return cudaErrorInvalidValue;
     const uint64_t want = (n_chains + 7) / 8;
     const unsigned grid = (unsigned)(want < (uint64_t)num_sms * 8 ? want : (uint64_t)num_sms * 8);
-    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n);
+    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp);
     return cudaGetLastError();
 }
 

@@ -60,6 +60,25 @@ struct ScanOut {
     uint64_t base;                  // global position of shard byte 0
     uint64_t *scratch;              // MODE_EMIT_OPT: q slots per chain
     uint32_t q;
+    // MODE_EMIT_OPT, staged kernel, when the main region starts the list
+    // (NULL = off): each CTA publishes its match total in tile_state
+    // [blockIdx.x] (decoupled look-back) and writes the end offset of each of
+    // its chains into chain_end_w -- the offset scan runs inside the scan
+    unsigned long long *tile_state;
+    uint64_t *chain_end_w;
+};
+
+// Decoupled look-back words: 2-bit flag (aggregate / inclusive prefix) + value.
+static constexpr uint64_t LB_AGG = 1ull << 62, LB_INC = 2ull << 62, LB_VAL = (1ull << 62) - 1;
+
+// Where k_gather finds chain offsets when the staged kernel computed them:
+// main chains from chain_end; the (few) tail chains behind the main total,
+// which is the last staged CTA's inclusive look-back word.
+struct TailPlace {
+    const unsigned long long *tile_state;  // NULL: chain_end holds every chain (k_offsets ran)
+    uint64_t n_tiles;                      // staged CTAs
+    uint64_t tail_c0, tail_n;              // tail chains (global ids), tail_n <= 256
+    uint64_t cap;
 };
 
 // Geometry of the TMA-staged main region.
@@ -107,9 +126,10 @@ size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
 // Single-pass list mode helpers: k_gather copies every chain's scratch slot
 // to its final position (or lists the chain when it overflowed); k_rewalk
 // re-scans the listed chains in MODE_EMIT.
-cudaError_t launch_gather(const uint64_t *counts, const uint64_t *chain_end, uint64_t n_chains,
-                          const uint64_t *scratch, uint32_t q, uint64_t *out, const ac_result *res,
-                          uint64_t *list, unsigned int *list_n, int num_sms, cudaStream_t stream);
+cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t n_chains,
+                          const uint64_t *scratch, uint32_t q, uint64_t *out, ac_result *res,
+                          uint64_t *list, unsigned int *list_n, const TailPlace &tp, int num_sms,
+                          cudaStream_t stream);
 cudaError_t launch_rewalk(uint32_t entry_bytes, uint32_t tier, const uint8_t *text, uint64_t n_total,
                           const SttView &st, const Region &a, const Region &b, const StagedGeom &g,
                           const ScanOut &so, const uint64_t *list, const unsigned int *list_n, size_t smem_stt,

@@ -42,7 +42,8 @@ def gpu_keys(stt, text_np: np.ndarray, **kw) -> np.ndarray:
     if c:  # the two-pass list mode and a forced-overflow single pass agree bit for bit
         _, r2 = ac.match(stt, t, two_pass=True, **kw)
         _, r3 = ac.match(stt, t, scratch_slots=2, **kw)  # most chains overflow -> k_rewalk
-        assert torch.equal(r2, recs) and torch.equal(r3, recs)
+        _, r4 = ac.match(stt, t, two_pass=2, **kw)  # single pass with the separate offset scan
+        assert torch.equal(r2, recs) and torch.equal(r3, recs) and torch.equal(r4, recs)
     assert cnt == c
     return recs.cpu().numpy()
 
