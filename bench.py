@@ -2,8 +2,9 @@
 """bench.py -- input-text Gbps of the Aho-Corasick matching scan on B200.
 
 One step = one pass of the whole hot path over one
-shard of synthetic text: ac_match_async in list mode (count scan -> chained
-offset scan -> emitting scan, canonical list written to HBM), plus the
+shard of synthetic text: ac_match_async in list mode (single emitting scan
+into per-chain scratch slots with the chain offsets computed in its epilogue
+-> gather into the canonical list in HBM -> overflow re-walk), plus the
 count all-reduce across ranks when N > 1.  The STT build and the host->device
 copy of the text are outside the timed region, as in the paper.
 
@@ -279,12 +280,18 @@ def run_ours(args):
     dom = max(kern, key=lambda k: k["ms"])
     hbm, hbm_src, pk = peaks()
     traffic = None
+    issue = None
     tf = ROOT / "profiles" / "traffic.json"
     if tf.exists():
-        traffic = json.loads(tf.read_text()).get(f"{args.config}/{args.mode}/{dom['name']}")
+        tj = json.loads(tf.read_text())
+        traffic = tj.get(f"{args.config}/{args.mode}/{dom['name']}")
+        issue = tj.get(f"{args.config}/{args.mode}/{dom['name']}/issue_active")
     achieved = dom["alg_bytes"] / (dom["ms"] * 1e-3) / 1e9
     roof = {"bound": "hbm", "kernel": dom["name"], "achieved": achieved, "peak": hbm, "unit": "GB/s",
             "frac": achieved / hbm, "traffic": traffic, "peak_source": hbm_src,
+            # what actually binds this kernel (ncu, same command): the SM issue
+            # slots -- fraction of cycles a warp scheduler issued an instruction
+            "sm_issue_active_frac": issue,
             "alg_bytes_per_launch": dom["alg_bytes"]}
 
     line = {

@@ -50,7 +50,9 @@ def build(force: bool = False, verbose: bool = False) -> Path:
 
     def compile_one(src: Path) -> Path:
         obj = OBJ / (src.name + ".o")
-        cmd = [nvcc(), *CFLAGS, *extra, f"-I{INCLUDE}", f"-I{CSRC}", "-c", str(src), "-o", str(obj)]
+        # AC_EXTRA_NVCC_FLAGS: experiment switches (e.g. -DAC_TEXT_EVICT_NORMAL), empty by default
+        exp = os.environ.get("AC_EXTRA_NVCC_FLAGS", "").split()
+        cmd = [nvcc(), *CFLAGS, *extra, *exp, f"-I{INCLUDE}", f"-I{CSRC}", "-c", str(src), "-o", str(obj)]
         if verbose:
             print(" ".join(cmd), flush=True)
         subprocess.check_call(cmd)

@@ -586,11 +586,20 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
             : "memory");
     } while (!done);
 }
-// The text is streamed exactly once: its TMA loads carry an L2 evict-first
-// policy so they do not push the automaton (L1/L2-resident tiers) out of L2.
-__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+// L2 policy of the text's TMA loads.  The text is streamed once, so for the
+// tiers whose automaton lives in L2 (GLOBAL, HYBRID) its loads are
+// evict-first: they must not push the STT out (C3: count 2,251 -> 2,860 Gbps).
+// For the shared-memory tiers it is evict-normal: a 16-byte-wide box uses half
+// of each 32-B sector and the next box the other half, so evict-first text
+// lines are re-read from DRAM (C2 list scan, ncu: 839 MB DRAM reads vs 341 MB,
+// 1.3 % slower).
+template <int TIER>
+__device__ __forceinline__ uint64_t text_l2_policy() {
     uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    if constexpr (TIER == AC_TIER_GLOBAL || TIER == AC_TIER_HYBRID)
+        asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    else
+        asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
     return pol;
 }
 __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y, uint64_t *bar,
@@ -734,7 +743,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     const bool tma_halo = (uint64_t)nh0 * W <= L;  // the halo window lies inside the next chain
     const uint32_t nh = tma_halo ? nh0 : 0;
     const uint32_t m = idle ? 0u : nh + (uint32_t)(L / W);
-    const uint64_t pol = l2_evict_first_policy();
+    const uint64_t pol = text_l2_policy<TIER>();
 
     auto issue = [&](uint32_t j) {
         const uint32_t slot = j % NST;

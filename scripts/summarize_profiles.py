@@ -73,7 +73,18 @@ def main(tag: str = "r01"):
         m = emit[-1]["metrics"]
         rd = float(m["dram__bytes_read.sum"]["value"]) * (1e6 if m["dram__bytes_read.sum"]["unit"] == "Mbyte" else 1e9)
         wr = float(m["dram__bytes_write.sum"]["value"]) * (1e6 if m["dram__bytes_write.sum"]["unit"] == "Mbyte" else 1e9)
-        json.dump({"c2/list/k_scan_staged(emit1)": int(rd + wr)}, open(PROF / "traffic.json", "w"), indent=1)
+        ia = float(m["smsp__issue_active.avg.pct_of_peak_sustained_active"]["value"]) / 100
+        json.dump({"c2/list/k_scan_staged(emit1)": int(rd + wr),
+                   "c2/list/k_scan_staged(emit1)/issue_active": round(ia, 4)}, open(PROF / "traffic.json", "w"), indent=1)
+    rep = OUT / "prof_c2_list.ncu-rep"
+    if rep.exists():  # the list-mode step's kernels (count scan, emitting scan, gather)
+        h, u, rows = ncu_raw(rep)
+        caps = [{"kernel": r[h.index("Kernel Name")],
+                 "metrics": {k: {"value": r[h.index(k)], "unit": u[h.index(k)]} for k in KEYS if k in h}}
+                for r in rows]
+        json.dump({"capture": "ncu --set full --clock-control none --import-source on -k regex:'k_scan_staged|k_gather', "
+                              "scripts/prof_target.py --config c2 --reps 2 (count scan, then list-mode steps)",
+                   "launches": caps}, open(PROF / f"{tag}_ncu_list_c2.json", "w"), indent=1)
     sweeps = {}
     for p in sorted(OUT.glob("sweep_*.jsonl")):
         sweeps[p.stem] = [json.loads(l) for l in open(p) if l.strip()]
