@@ -13,3 +13,4 @@ done
 timeout 600 python scripts/sweep.py --config c2 --variants 7 --global-kernel --tiers compact,global > gpurun_out/sweep_c2.jsonl 2> gpurun_out/sweep_c2.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 3 --warmup 1 --no-e2e --no-cpu-baseline > gpurun_out/ncu_bench.out 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_scan_staged -s 2 -c 2 -o gpurun_out/prof_c2_full python scripts/prof_target.py --config c2 --reps 2 > gpurun_out/ncu_full.out 2>&1
+bash scripts/gpu_ncu_list.sh
