@@ -164,7 +164,9 @@ typedef struct {
                               the text pointer is 16-byte aligned, else by
                               a separate offset scan); 1 = count pass + emit
                               pass (ablation / fallback); 2 = single pass
-                              with the separate offset scan (ablation)     */
+                              with the separate offset scan (ablation);
+                              3 = single pass with 8-byte scratch records
+                              (ablation of the 4-byte narrow records)      */
     uint32_t stride;       /* 0 = the table's default, 1 = force one byte
                               per lookup even if a two-byte table exists     */
     uint32_t n_events;     /* pairs available in `events`                    */

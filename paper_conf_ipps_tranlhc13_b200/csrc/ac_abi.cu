@@ -346,6 +346,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         ac_status rc = side_stream(h->device, &side);
         if (rc != AC_OK) return rc;
     }
+    uint32_t nm_bits = 0;  // narrow scratch records in the staged kernel (list mode, set below)
     auto scan = [&](int mode, const char *gname, const char *sname) -> ac_status {
         if (any_global) {
             cudaStream_t gs = stream;
@@ -361,7 +362,9 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         }
         if (g.n_chains) {
             pre();
-            AC_CUDA(launch_scan_staged(mode, eb, tier_s, variant, tmap, d_text + g.m0, ss, g, so, smem_s, stream),
+            ScanOut sso = so;
+            if (mode == MODE_EMIT_OPT) sso.nbits = nm_bits;
+            AC_CUDA(launch_scan_staged(mode, eb, tier_s, variant, tmap, d_text + g.m0, ss, g, sso, smem_s, stream),
                     sname);
             post(sname);
         }
@@ -395,6 +398,17 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     so.tile_state = lb;
     so.chain_end_w = chain_end;
     TailPlace tp{lb, n_lb, rb.chain0, rb.n_chains, cap};
+    // narrow scratch records for the staged kernel's deferred emission (one
+    // chain per lane, 16-bit table, one byte per lookup): offset in chain and
+    // pattern id must share 32 bits.  Off for the two-pass ablation.
+    NarrowMain nm{0, g.chain0, g.n_chains, base + g.m0, g.chain_len};
+    if (!two_pass && g.n_chains && cfg.k == 1 && eb == 2 && !ss.stt2 && !(opts && opts->two_pass == 3)) {
+        uint32_t pid_bits = 1, off_bits = 1;
+        while ((1ull << pid_bits) < h->host.n_patterns) pid_bits++;
+        while ((1ull << off_bits) < g.chain_len) off_bits++;
+        if (pid_bits + off_bits <= 32) nm.nbits = pid_bits;
+    }
+    nm_bits = nm.nbits;
     so.chain_counts = counts;
     so.chain_end = chain_end;
     // single pass: each chain keeps its first q records in a scratch slot
@@ -433,7 +447,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             post("k_offsets");
         }
         pre();
-        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, tp,
+        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, tp, nm,
                               h->num_sms, stream),
                 "k_gather");
         post("k_gather");

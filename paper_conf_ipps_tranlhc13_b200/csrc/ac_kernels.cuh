@@ -398,6 +398,15 @@ __device__ __forceinline__ void st_global_if(const uint64_t *base, int32_t k, ui
         : "memory");
 }
 
+// Predicated 4-byte global store to base[k] (narrow scratch records).
+__device__ __forceinline__ void st_global32_if(const uint32_t *base, int32_t k, uint32_t v, bool pred) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ne.u32 p, %3, 0;\n\t"
+        "mad.wide.s32 a, %1, 4, %0;\n\t@p st.global.u32 [a], %2;\n\t}" ::"l"(base),
+        "r"(k), "r"(v), "r"((uint32_t)pred)
+        : "memory");
+}
+
 __device__ __forceinline__ uint32_t byte_of(const uint4 &v, int bb) {
     const uint32_t w = (bb >> 2) == 0 ? v.x : (bb >> 2) == 1 ? v.y : (bb >> 2) == 2 ? v.z : v.w;
     return __byte_perm(w, 0, 0x4440 | (bb & 3));  // one PRMT: zero-extended byte bb & 3
@@ -883,57 +892,73 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                     if (!live[0]) fm = 0;
                     if constexpr (MODE == MODE_EMIT_OPT) {
                         // record k of the chain goes to slot last - k (if k < q);
-                        // nk = -k keeps the address one IMAD.WIDE away
+                        // nk = -k keeps the address one IMAD.WIDE away.  Wide
+                        // records are the final 8-byte keys; narrow ones (so.nbits
+                        // > 0) are (offset in chain << nbits | pattern), 4 bytes,
+                        // widened by k_gather -- half the scratch traffic
                         const uint64_t *const last = reinterpret_cast<const uint64_t *>(wp[0]);
+                        const uint32_t *const last32 = reinterpret_cast<const uint32_t *>(wp[0] + 4);
                         int32_t nk = -(int32_t)cnt[0];
                         int32_t nq = -(int32_t)so.q;
-                        // COMPACT output-table base: made opaque so that it (and
-                        // nq) stay in registers instead of being re-derived from
-                        // constants in every iteration (measured: ~10 uniform-
-                        // datapath instructions per iteration otherwise)
+                        // COMPACT output-table base kept in a register (ptxas
+                        // may still re-derive nq from the constant bank)
                         uint32_t ob = smem_u32(s_stt) + st.c_out_x0;
                         asm volatile("" : "+r"(ob), "+r"(nq));
+                        const uint32_t nb = so.nbits;
+                        const uint32_t kn = ((uint32_t)col0 + (uint32_t)q * 16u) << nb;  // chunk offset, narrow
                         // A warp-uniform trip count (the most flags any lane
                         // holds) instead of a divergent while-any loop: no
                         // reconvergence bookkeeping, predicated body.
                         const uint32_t iters = __reduce_max_sync(0xffffffffu, (uint32_t)__popc(fm));
-                        for (uint32_t it = 0; it < iters; ++it) {
-                            uint32_t bb;  // highest flagged byte left (0xffffffff if none)
-                            asm("bfind.u32 %0, %1;" : "=r"(bb) : "r"(fm));
-                            const uint32_t act = fm != 0;
-                            fm &= ~(1u << (bb & 31u));
-                            const uint32_t i = bb >> 1;
-                            const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
-                            const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
-                            const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
-                            const uint32_t pr = (i & 4) ? b1 : b0;
-                            const uint32_t x = __byte_perm(pr, 0, (bb & 1) ? 0x4410 : 0x4432);
-                            uint2 o;
-                            if constexpr (TIER == AC_TIER_COMPACT) {
-                                o = make_uint2(0u, 0u);
-                                asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t}"
-                                    : "+r"(o.x), "+r"(o.y)
-                                    : "r"(ob + x * 8u), "r"(act));
-                            } else {
-                                o = out_info_pred<E, TIER, true>(s_stt, st, x, act);
+                        auto emit_loop = [&](auto narrow_tag) {
+                            constexpr bool NARROW = decltype(narrow_tag)::value;
+                            for (uint32_t it = 0; it < iters; ++it) {
+                                uint32_t bb;  // highest flagged byte left (0xffffffff if none)
+                                asm("bfind.u32 %0, %1;" : "=r"(bb) : "r"(fm));
+                                const uint32_t act = fm != 0;
+                                fm &= ~(1u << (bb & 31u));
+                                const uint32_t i = bb >> 1;
+                                const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
+                                const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
+                                const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
+                                const uint32_t pr = (i & 4) ? b1 : b0;
+                                const uint32_t x = __byte_perm(pr, 0, (bb & 1) ? 0x4410 : 0x4432);
+                                uint2 o;
+                                if constexpr (TIER == AC_TIER_COMPACT) {
+                                    o = make_uint2(0u, 0u);
+                                    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%2];\n\t}"
+                                        : "+r"(o.x), "+r"(o.y)
+                                        : "r"(ob + x * 8u), "r"(act));
+                                } else {
+                                    o = out_info_pred<E, TIER, true>(s_stt, st, x, act);
+                                }
+                                uint32_t c = o.y;
+                                if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
+                                    c = __ldg(st.out_off + x + 1) - __ldg(st.out_off + x);
+                                // wide key = (start << 24) | pid with start = chunk start +
+                                // bb: bb << 24 | pid < 2^32 (bb <= 15, pid < 2^24) is added
+                                // to the chunk's key as ONE 32-bit addend; narrow: the same
+                                // with the chain-relative offset and nb pattern bits
+                                // (garbage, and never stored, in lanes with no flag left)
+                                const uint32_t add = NARROW ? (bb << nb) + kn : bb * (1u << 24);
+                                auto put = [&](int32_t k, uint32_t pid, bool pred) {
+                                    if constexpr (NARROW)
+                                        st_global32_if(last32, k, add + pid, pred);
+                                    else
+                                        st_global_if(last, k, kb[0] + (add + pid), pred);
+                                };
+                                put(nk, o.x, (c == 1u) & (nk > nq));
+                                if (__any_sync(0xffffffffu, c > 1u)) {  // multi-output states (rare)
+                                    for (uint32_t j = 0; j < c && c > 1u; ++j)
+                                        put(nk - (int32_t)j, __ldg(st.out_ids + o.x + c - 1 - j), nk - (int32_t)j > nq);
+                                }
+                                nk -= (int32_t)c;
                             }
-                            uint32_t c = o.y;
-                            if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
-                                c = __ldg(st.out_off + x + 1) - __ldg(st.out_off + x);
-                            // key = (start << 24) | pid with start = chunk start + bb:
-                            // bb << 24 | pid < 2^32 (bb <= 15, pid < 2^24) is added
-                            // to the chunk's key as ONE 32-bit addend (garbage, and
-                            // never stored, in lanes with no flag left)
-                            const uint32_t add = bb * (1u << 24);
-                            st_global_if(last, nk, kb[0] + (add + o.x), (c == 1u) & (nk > nq));
-                            if (__any_sync(0xffffffffu, c > 1u)) {  // multi-output states (rare)
-                                for (uint32_t j = 0; j < c && c > 1u; ++j)
-                                    st_global_if(last, nk - (int32_t)j,
-                                                 kb[0] + (add + __ldg(st.out_ids + o.x + c - 1 - j)),
-                                                 nk - (int32_t)j > nq);
-                            }
-                            nk -= (int32_t)c;
-                        }
+                        };
+                        if (nb)
+                            emit_loop(std::true_type{});
+                        else
+                            emit_loop(std::false_type{});
                         cnt[0] = (uint32_t)(-nk);
                     } else
                     while (__any_sync(0xffffffffu, fm)) {

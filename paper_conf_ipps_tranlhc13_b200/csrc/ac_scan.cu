@@ -132,7 +132,7 @@ static constexpr uint64_t kMaxTail = 256;
 __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ counts, uint64_t *chain_end,
                                                 uint64_t n_chains, const uint64_t *__restrict__ scratch, uint32_t q,
                                                 uint64_t *__restrict__ out, ac_result *res, uint64_t *list,
-                                                unsigned int *list_n, TailPlace tp) {
+                                                unsigned int *list_n, TailPlace tp, NarrowMain nm) {
     const int lane = threadIdx.x & 31;
     uint64_t main_total = 0;
     if (tp.tile_state) {
@@ -172,8 +172,26 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
             if (lane == 0) list[atomicAdd(list_n, 1u)] = c;
             continue;
         }
-        const uint64_t *src = scratch + c * q + (q - cnt);
         uint64_t *dst = out + end - cnt;
+        if (nm.nbits && c - nm.c0 < nm.n) {
+            // narrow records (offset << nbits | pid) packed at the slot's end
+            const uint32_t *src = reinterpret_cast<const uint32_t *>(scratch + (c + 1) * q) - cnt;
+            const uint64_t lo = nm.lo0 + (c - nm.c0) * nm.chain_len;  // chain's first byte
+            const uint32_t nb = nm.nbits, pm = (1u << nb) - 1u;
+            auto widen = [&](uint32_t r) { return ((lo + (r >> nb)) << 24) | (r & pm); };
+            uint64_t i = lane;
+            for (; i + 96 < cnt; i += 128) {
+                const uint32_t a = __ldg(src + i), b = __ldg(src + i + 32), d = __ldg(src + i + 64),
+                               e = __ldg(src + i + 96);
+                dst[i] = widen(a);
+                dst[i + 32] = widen(b);
+                dst[i + 64] = widen(d);
+                dst[i + 96] = widen(e);
+            }
+            for (; i < cnt; i += 32) dst[i] = widen(__ldg(src + i));
+            continue;
+        }
+        const uint64_t *src = scratch + c * q + (q - cnt);
         // four records in flight per lane before the stores
         uint64_t i = lane;
         for (; i + 96 < cnt; i += 128) {
@@ -190,13 +208,13 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
 
 cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t n_chains,
                           const uint64_t *scratch, uint32_t q, uint64_t *out, ac_result *res,
-                          uint64_t *list, unsigned int *list_n, const TailPlace &tp, int num_sms,
-                          cudaStream_t stream) {
+                          uint64_t *list, unsigned int *list_n, const TailPlace &tp, const NarrowMain &nm,
+                          int num_sms, cudaStream_t stream) {
     if (n_chains == 0) return cudaSuccess;
     if (tp.tile_state && tp.tail_n > kMaxTail) return cudaErrorInvalidValue;
     const uint64_t want = (n_chains + 7) / 8;
     const unsigned grid = (unsigned)(want < (uint64_t)num_sms * 8 ? want : (uint64_t)num_sms * 8);
-    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp);
+    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp, nm);
     return cudaGetLastError();
 }
 

@@ -60,6 +60,10 @@ struct ScanOut {
     uint64_t base;                  // global position of shard byte 0
     uint64_t *scratch;              // MODE_EMIT_OPT: q slots per chain
     uint32_t q;
+    // MODE_EMIT_OPT, staged kernel's deferred emission only: > 0 = narrow
+    // 4-byte scratch records (offset in chain << nbits | pattern), packed at
+    // the end of the chain's 8q-byte slot; 0 = 8-byte final keys
+    uint32_t nbits;
     // MODE_EMIT_OPT, staged kernel, when the main region starts the list
     // (NULL = off): each CTA publishes its match total in tile_state
     // [blockIdx.x] (decoupled look-back) and writes the end offset of each of
@@ -74,6 +78,14 @@ static constexpr uint64_t LB_AGG = 1ull << 62, LB_INC = 2ull << 62, LB_VAL = (1u
 // Where k_gather finds chain offsets when the staged kernel computed them:
 // main chains from chain_end; the (few) tail chains behind the main total,
 // which is the last staged CTA's inclusive look-back word.
+// Main-region chains whose scratch records are narrow (k_gather widens them).
+struct NarrowMain {
+    uint32_t nbits;       // 0 = every chain is wide
+    uint64_t c0, n;       // global ids of the main chains
+    uint64_t lo0;         // global position of main chain 0's first byte (base + m0)
+    uint64_t chain_len;   // L
+};
+
 struct TailPlace {
     const unsigned long long *tile_state;  // NULL: chain_end holds every chain (k_offsets ran)
     uint64_t n_tiles;                      // staged CTAs
@@ -128,8 +140,8 @@ size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
 // re-scans the listed chains in MODE_EMIT.
 cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t n_chains,
                           const uint64_t *scratch, uint32_t q, uint64_t *out, ac_result *res,
-                          uint64_t *list, unsigned int *list_n, const TailPlace &tp, int num_sms,
-                          cudaStream_t stream);
+                          uint64_t *list, unsigned int *list_n, const TailPlace &tp, const NarrowMain &nm,
+                          int num_sms, cudaStream_t stream);
 cudaError_t launch_rewalk(uint32_t entry_bytes, uint32_t tier, const uint8_t *text, uint64_t n_total,
                           const SttView &st, const Region &a, const Region &b, const StagedGeom &g,
                           const ScanOut &so, const uint64_t *list, const unsigned int *list_n, size_t smem_stt,
