@@ -267,7 +267,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
 
     // --- geometry: [head | main (staged) | tail] or a single global region
     Region ra{0, 0, kGlobalTailChain, 0, 0}, rb{0, 0, kGlobalTailChain, 0, 0};
-    StagedGeom g{0, 0, 0, 0, 0};
+    StagedGeom g{0, 0, 0, 0, 0, 0};
     CUtensorMap tmap;
     if (kernel == AC_KERNEL_STAGED) {
         const uint64_t W = (uint64_t)cfg.width, R = (uint64_t)cfg.warps * 32 * cfg.k;
@@ -294,6 +294,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             g.n_chains = n_main;
             g.chain0 = ra.n_chains;
             g.n_readable = n_total - head;
+            g.text_evict_first = (tier_s == AC_TIER_GLOBAL || tier_s == AC_TIER_HYBRID) ? 1u : 0u;
             PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
             if (!enc) {
                 set_error("cuTensorMapEncodeTiled unavailable from the driver");

@@ -595,17 +595,17 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
             : "memory");
     } while (!done);
 }
-// L2 policy of the text's TMA loads.  The text is streamed once, so for the
-// tiers whose automaton lives in L2 (GLOBAL, HYBRID) its loads are
-// evict-first: they must not push the STT out (C3: count 2,251 -> 2,860 Gbps).
-// For the shared-memory tiers it is evict-normal: a 16-byte-wide box uses half
-// of each 32-B sector and the next box the other half, so evict-first text
-// lines are re-read from DRAM (C2 list scan, ncu: 839 MB DRAM reads vs 341 MB,
-// 1.3 % slower).
-template <int TIER>
-__device__ __forceinline__ uint64_t text_l2_policy() {
+// L2 policy of the text's TMA loads (chosen by the planner, StagedGeom).
+// The text is streamed once: where the automaton lives in L2 (GLOBAL,
+// HYBRID) its loads are evict-first so they do not push the STT out (C3:
+// count 2,251 -> 2,860 Gbps).  For the shared-memory tiers they are
+// evict-normal: a 16-byte box uses half of each 32-B sector and the next box
+// the other half, so evict-first text lines are re-read from DRAM (C2 list
+// scan, ncu: 839 MB DRAM reads vs 341 MB; step 0.5324 vs 0.5294 ms; with
+// 32-byte boxes evict-first was also slower, 0.697 vs 0.683 ms).
+__device__ __forceinline__ uint64_t text_l2_policy(uint32_t evict_first) {
     uint64_t pol;
-    if constexpr (TIER == AC_TIER_GLOBAL || TIER == AC_TIER_HYBRID)
+    if (evict_first)
         asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
     else
         asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
@@ -752,7 +752,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     const bool tma_halo = (uint64_t)nh0 * W <= L;  // the halo window lies inside the next chain
     const uint32_t nh = tma_halo ? nh0 : 0;
     const uint32_t m = idle ? 0u : nh + (uint32_t)(L / W);
-    const uint64_t pol = text_l2_policy<TIER>();
+    const uint64_t pol = text_l2_policy(g.text_evict_first);
 
     auto issue = [&](uint32_t j) {
         const uint32_t slot = j % NST;

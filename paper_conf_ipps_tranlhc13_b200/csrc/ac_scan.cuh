@@ -100,6 +100,7 @@ struct StagedGeom {
     uint64_t n_chains;     // full chains in the main region
     uint64_t chain0;       // global index of main chain 0
     uint64_t n_readable;   // bytes readable from the main-region pointer (halo bound)
+    uint32_t text_evict_first;  // L2 policy of the text's TMA loads (see text_l2_policy)
 };
 
 struct StagedConfig {
