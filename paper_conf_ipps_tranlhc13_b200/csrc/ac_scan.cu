@@ -173,36 +173,33 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
             continue;
         }
         uint64_t *dst = out + end - cnt;
+        // every load of a batch is issued before its stores (predicated, not
+        // a remainder loop): a typical chain (~100 records) is one round trip
+        constexpr int B = 8;
         if (nm.nbits && c - nm.c0 < nm.n) {
             // narrow records (offset << nbits | pid) packed at the slot's end
             const uint32_t *src = reinterpret_cast<const uint32_t *>(scratch + (c + 1) * q) - cnt;
             const uint64_t lo = nm.lo0 + (c - nm.c0) * nm.chain_len;  // chain's first byte
             const uint32_t nb = nm.nbits, pm = (1u << nb) - 1u;
-            auto widen = [&](uint32_t r) { return ((lo + (r >> nb)) << 24) | (r & pm); };
-            uint64_t i = lane;
-            for (; i + 96 < cnt; i += 128) {
-                const uint32_t a = __ldg(src + i), b = __ldg(src + i + 32), d = __ldg(src + i + 64),
-                               e = __ldg(src + i + 96);
-                dst[i] = widen(a);
-                dst[i + 32] = widen(b);
-                dst[i + 64] = widen(d);
-                dst[i + 96] = widen(e);
+            for (uint64_t i = lane; i < cnt; i += 32 * B) {
+                uint32_t r[B];
+#pragma unroll
+                for (int u = 0; u < B; u++) r[u] = i + 32 * u < cnt ? __ldg(src + i + 32 * u) : 0u;
+#pragma unroll
+                for (int u = 0; u < B; u++)
+                    if (i + 32 * u < cnt) dst[i + 32 * u] = ((lo + (r[u] >> nb)) << 24) | (r[u] & pm);
             }
-            for (; i < cnt; i += 32) dst[i] = widen(__ldg(src + i));
             continue;
         }
         const uint64_t *src = scratch + c * q + (q - cnt);
-        // four records in flight per lane before the stores
-        uint64_t i = lane;
-        for (; i + 96 < cnt; i += 128) {
-            const uint64_t a = __ldg(src + i), b = __ldg(src + i + 32), d = __ldg(src + i + 64),
-                           e = __ldg(src + i + 96);
-            dst[i] = a;
-            dst[i + 32] = b;
-            dst[i + 64] = d;
-            dst[i + 96] = e;
+        for (uint64_t i = lane; i < cnt; i += 32 * B) {
+            uint64_t r[B];
+#pragma unroll
+            for (int u = 0; u < B; u++) r[u] = i + 32 * u < cnt ? __ldg(src + i + 32 * u) : 0ull;
+#pragma unroll
+            for (int u = 0; u < B; u++)
+                if (i + 32 * u < cnt) dst[i + 32 * u] = r[u];
         }
-        for (; i < cnt; i += 32) dst[i] = __ldg(src + i);
     }
 }
 
