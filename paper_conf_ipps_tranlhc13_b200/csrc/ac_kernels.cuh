@@ -833,36 +833,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                 // (COMPACT counting keeps its predicated per-byte count: measured faster)
                 constexpr bool kDeferred = STRIDE == 1 && K == 1 && sizeof(E) == 2 &&
                                            (TIER != AC_TIER_COMPACT || MODE == MODE_EMIT || MODE == MODE_EMIT_OPT);
-                // Deferred-by-rewalk for 32-bit tables: measured SLOWER on C3
-                // (count 3.81 -> 4.95 ms, the L1-bound walk lost its overlap),
-                // so it is compiled out; kept for the record and for experiments.
-                constexpr bool kRewalk = false && STRIDE == 1 && K == 1 && sizeof(E) == 4;
-                if constexpr (kRewalk) {
-                    // 32-bit states do not pack into a register history: walk
-                    // the chunk recording only the flag mask, and re-walk it
-                    // from its start state in the (rare) lanes that matched.
-                    uint32_t fm = 0, st0 = s[0];
-                    const uint32_t s_start = st0;
-#pragma unroll
-                    for (int bb = 15; bb >= 0; --bb) {
-                        const uint32_t e = next_entry<E, TIER>(s_stt, st, st0, s_cmap[byte_of(v[0], bb)]);
-                        st0 = e & EntryBits<E>::MASK;
-                        fm |= (e >> 31) << bb;
-                    }
-                    s[0] = st0;
-                    if (!live[0]) fm = 0;
-                    if (__any_sync(0xffffffffu, fm) && fm) {
-                        uint32_t x = s_start;
-#pragma unroll
-                        for (int bb = 15; bb >= 0; --bb) {
-                            const uint32_t e = next_entry<E, TIER>(s_stt, st, x, s_cmap[byte_of(v[0], bb)]);
-                            x = e & EntryBits<E>::MASK;
-                            if (e >> 31)
-                                emit_outputs<E, TIER, MODE>(x, kb[0] + ((uint64_t)bb << 24), cnt[0], wp[0], s_stt,
-                                                            st, so);
-                        }
-                    }
-                } else if constexpr (kDeferred) {
+                // (a deferred-by-rewalk variant for 32-bit tables -- flag mask only,
+                // re-walk the chunk in lanes that matched -- was measured slower on
+                // C3, count 3.81 -> 4.95 ms: the L1-bound walk lost its overlap)
+                if constexpr (kDeferred) {
                     // Deferred emission: walk the 16 bytes recording the
                     // flag bits and the (16-bit) states in registers, then
                     // emit in a warp-uniform loop that runs max-over-lanes
