@@ -268,12 +268,15 @@ def run_ours(args):
         acc += [a.elapsed_time(b) for a, b in pairs]
     kms = acc / reps
     out_bytes = 8 * count if args.mode == "list" else 0
+    # single pass: the scan writes each record to its chain's scratch slot
+    # (4 B narrow / 8 B), the gather reads it back and writes the 8-B key
+    rec = ac.last_scratch_record_bytes() if args.mode == "list" else 0
     kern = []
     for nm, t in zip(names, kms):
         if "scan" in nm:
-            byts = n + (out_bytes if "emit" in nm else 0)
+            byts = n + (rec * count if "emit1" in nm else out_bytes if "emit" in nm else 0)
         elif "gather" in nm:
-            byts = 2 * out_bytes  # every record read from its scratch slot and written once
+            byts = (rec + 8) * count
         else:
             byts = 0  # offset scan / overflow re-walk: latency-bound bookkeeping
         kern.append({"name": nm, "ms": float(t), "share": float(t / ms), "alg_bytes": int(byts)})

@@ -243,6 +243,10 @@ ac_status ac_match_segments(const ac_stt *stt, const uint8_t *d_text, const uint
  * and the name of launch i (NULL if out of range). */
 uint32_t ac_last_launch_count(void);
 const char *ac_last_launch_name(uint32_t i);
+/* Bytes per scratch record of the last list-mode ac_match_async on this
+ * thread: 4 (narrow: offset in chain and pattern id share 32 bits), 8, or 0
+ * (count mode / two-pass mode: no scratch).  For traffic accounting. */
+uint32_t ac_last_scratch_record_bytes(void);
 
 /* End-to-end entry with HOST buffers: copies h_text[0,n) to the device,
  * scans it, copies the count and (if h_out != NULL) the canonical list back

@@ -33,7 +33,7 @@ TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global", 4: "compact"}
 
 EXPORTED = [
     "ac_build", "ac_free", "ac_stt_query", "ac_stt_pattern_lengths", "ac_match", "ac_match_shard",
-    "ac_match_async", "ac_match_segments", "ac_last_launch_count", "ac_last_launch_name", "ac_match_host", "ac_compile", "ac_table_query",
+    "ac_match_async", "ac_match_segments", "ac_last_launch_count", "ac_last_launch_name", "ac_last_scratch_record_bytes", "ac_match_host", "ac_compile", "ac_table_query",
     "ac_table_export", "ac_table_export_compact", "ac_table_export_stride2", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
 ]
 
@@ -107,6 +107,8 @@ def lib():
         L.ac_last_launch_count.argtypes = []
         L.ac_last_launch_name.restype = ctypes.c_char_p
         L.ac_last_launch_name.argtypes = [_u32]
+        L.ac_last_scratch_record_bytes.restype = _u32
+        L.ac_last_scratch_record_bytes.argtypes = []
         L.ac_status_string.restype = ctypes.c_char_p
         L.ac_status_string.argtypes = [ctypes.c_int]
         L.ac_last_error.restype = ctypes.c_char_p
@@ -316,6 +318,11 @@ def last_launch_count() -> int:
 def last_launch_names() -> list[str]:
     L = lib()
     return [L.ac_last_launch_name(i).decode() for i in range(L.ac_last_launch_count())]
+
+
+def last_scratch_record_bytes() -> int:
+    """4 (narrow), 8 or 0: scratch bytes per record of the last list-mode call."""
+    return int(lib().ac_last_scratch_record_bytes())
 
 
 def version() -> str:

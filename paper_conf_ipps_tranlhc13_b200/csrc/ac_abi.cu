@@ -19,6 +19,7 @@ namespace acx {
 
 static thread_local std::string g_err;
 static thread_local uint32_t g_launches = 0;
+static thread_local uint32_t g_scratch_rec = 0;  // bytes per scratch record of the last list-mode call
 static thread_local const char *g_names[16];
 
 void set_error(const std::string &msg) { g_err = msg; }
@@ -208,6 +209,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
                              uint64_t base, ac_match_t *d_out, uint64_t cap, ac_result *d_res, cudaStream_t stream,
                              const ac_match_opts *opts) {
     g_launches = 0;
+    g_scratch_rec = 0;
     if (!h || !d_res || (!d_text && n_owned + n_halo > 0)) {
         set_error("NULL stt, result or text");
         return AC_ERR_INVALID_ARG;
@@ -410,6 +412,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         if (pid_bits + off_bits <= 32) nm.nbits = pid_bits;
     }
     nm_bits = nm.nbits;
+    g_scratch_rec = two_pass ? 0u : nm.nbits ? 4u : 8u;
     so.chain_counts = counts;
     so.chain_end = chain_end;
     // single pass: each chain keeps its first q records in a scratch slot
@@ -688,6 +691,7 @@ const char *ac_status_string(ac_status s) {
 const char *ac_last_error(void) { return g_err.c_str(); }
 const char *ac_version(void) { return "libac 0.1 sm_100a (TMA-staged + global-only scans)"; }
 uint32_t ac_last_launch_count(void) { return g_launches; }
+uint32_t ac_last_scratch_record_bytes(void) { return g_scratch_rec; }
 const char *ac_last_launch_name(uint32_t i) { return i < g_launches && i < 16 ? g_names[i] : nullptr; }
 
 ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n, const ac_build_opts *opts,
