@@ -194,6 +194,16 @@ def test_chunking_invariance_staged(chain):
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, chain_bytes=chain), oracle_keys(o, w.text))
 
 
+def test_in_kernel_offsets_more_ctas_than_sms():
+    # 16-byte chains over 8 MiB: 512 staged CTAs (> 148 SMs, not all
+    # co-resident) chain their totals through the in-kernel look-back; a
+    # ragged tail of 13 bytes goes to the side-stream kernel
+    w = synth.make("c1", n=(8 << 20) + 13)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=4, chain_bytes=16), oracle_keys(o, w.text))
+
+
 @pytest.mark.parametrize("chain", [1, 7, 16, 64, 1000, 1 << 20])
 def test_chunking_invariance_global(chain):
     w = synth.make("c1", n=(1 << 18) + 3)
