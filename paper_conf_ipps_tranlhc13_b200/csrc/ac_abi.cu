@@ -40,7 +40,7 @@ static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slot
 static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slots (32 KB ring)
 // COMPACT budget used by ac_compile (no device): B200's 227 KB opt-in shared
 // memory minus the lean staged variant's ring and bookkeeping (= stt_budget)
-#define kDefaultCompactBudget (232448 - staged_smem_bytes(staged_variant(kLeanVariant), 0) - 1024)
+#define kDefaultCompactBudget (232448 - staged_smem_bytes(staged_variant(kLeanVariant), 0) - 128)
 // Below ~32 MiB the staged kernel cannot fill 148 SMs x 1024 chains with
 // chains of >= 256 B; the global kernel's shorter chains win (C1: 1 MiB list
 // 0.037 ms global vs 0.052 ms staged).
@@ -139,7 +139,7 @@ static ac_status check_device(int device, cudaDeviceProp *prop) {
 // Shared memory left for STT rows by a staged variant (v >= 1) or by the
 // global-only kernel (v == 0).
 static size_t stt_budget(const ac_stt *h, int v) {
-    const size_t fixed = (v ? staged_smem_bytes(staged_variant(v), 0) : 256) + 1024;  // + static smem / slack
+    const size_t fixed = (v ? staged_smem_bytes(staged_variant(v), 0) : 256) + 128;  // + static smem (k_rewalk: 64 B)
     return h->smem_optin > fixed ? h->smem_optin - fixed : 0;
 }
 

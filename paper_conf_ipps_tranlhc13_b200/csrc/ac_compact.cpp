@@ -77,47 +77,76 @@ bool compact_table(ac_table &t, size_t budget) {
     for (uint32_t s = 0; s < S; s++) maxd = std::max(maxd, t.depth[s]);
     // the deepest dense prefix that fits (the size is not monotonic in d:
     // shallow prefixes force many states with > 2 exceptions to be dense)
-    int best = -1;
-    for (uint32_t d = 0; d <= maxd; d++)
-        if (compact_bytes_for(t, d, nullptr, nullptr, nullptr) <= budget) best = (int)d;
-    if (best < 0) return false;
-    // Fill the rest of the budget with deeper states, most patterns below
-    // them first: a state that prefixes many patterns is a common string
-    // (the patterns are words of the text), so it is visited often,
-    // and making it dense also lets its descendants' records fall back on
-    // it (fewer exceptions, fewer exception-forced dense states).  Measured
-    // on the C2 text (simulated walk): sparse visits 48 % -> 32 %.
+    // Dense set = the depth-<= d prefix + the first k of the deeper states
+    // ordered by how many patterns they prefix (most first): a state that
+    // prefixes many patterns is a common string (the patterns are words of
+    // the text), so it is visited often, and making it dense also lets
+    // its descendants' records fall back on it (fewer exceptions, fewer
+    // exception-forced dense states -- the size is not monotonic in d or k).
+    // Take the deepest prefix that fits and fill the rest of the budget; if
+    // no prefix fits, the (d, k) with the most dense states that does.
+    // Measured on the C2 text (simulated walk): sparse visits 48 % -> 34 %.
+    std::vector<uint32_t> parent(S, 0), below(S, 0);
+    for (uint32_t s = 0; s < S; s++)
+        for (uint32_t c = 0; c < C; c++) {
+            uint16_t e;
+            std::memcpy(&e, &t.stt[((size_t)s * stride + c) * 2], 2);
+            const uint32_t u = e & 0x7fffu;
+            if (u && t.depth[u] == t.depth[s] + 1) parent[u] = s;  // the goto edge (unique)
+        }
+    for (uint32_t s = 1; s < S; s++)  // patterns ending exactly at s
+        for (uint32_t j = t.out_off[s]; j < t.out_off[s + 1]; j++) below[s] += t.lens[t.out_ids[j]] == t.depth[s];
+    for (uint32_t s = S - 1; s > 0; s--) below[parent[s]] += below[s];  // BFS order: children after parents
     std::vector<uint8_t> seed(S, 0);
-    {
-        std::vector<uint32_t> parent(S, 0), below(S, 0);
-        for (uint32_t s = 0; s < S; s++)
-            for (uint32_t c = 0; c < C; c++) {
-                uint16_t e;
-                std::memcpy(&e, &t.stt[((size_t)s * stride + c) * 2], 2);
-                const uint32_t u = e & 0x7fffu;
-                if (u && t.depth[u] == t.depth[s] + 1) parent[u] = s;  // the goto edge (unique)
-            }
-        for (uint32_t s = 1; s < S; s++)  // patterns ending exactly at s
-            for (uint32_t j = t.out_off[s]; j < t.out_off[s + 1]; j++) below[s] += t.lens[t.out_ids[j]] == t.depth[s];
-        for (uint32_t s = S - 1; s > 0; s--) below[parent[s]] += below[s];  // BFS order: children after parents
-        std::vector<uint32_t> cand;
+    std::vector<uint32_t> cand;
+    auto candidates = [&](uint32_t d) {
+        cand.clear();
         for (uint32_t s = 1; s < S; s++)
-            if (t.depth[s] > (uint32_t)best) cand.push_back(s);
+            if (t.depth[s] > d) cand.push_back(s);
         std::stable_sort(cand.begin(), cand.end(), [&](uint32_t a, uint32_t b) {
             return below[a] != below[b] ? below[a] > below[b] : t.depth[a] < t.depth[b];
         });
-        auto fits = [&](size_t k) {
-            std::fill(seed.begin(), seed.end(), 0);
-            for (size_t i = 0; i < k; i++) seed[cand[i]] = 1;
-            return compact_bytes_for(t, (uint32_t)best, &seed, nullptr, nullptr) <= budget;
-        };
-        size_t lo = 0, hi = cand.size();  // largest k that fits (size is close to monotone in k)
+    };
+    uint32_t nd_try = 0;
+    auto fits = [&](uint32_t d, size_t k) {
+        std::fill(seed.begin(), seed.end(), 0);
+        for (size_t i = 0; i < k; i++) seed[cand[i]] = 1;
+        return compact_bytes_for(t, d, &seed, nullptr, &nd_try) <= budget;
+    };
+    // the largest fitting k, given that k = lo fits (bisection; near-monotone)
+    auto widest = [&](uint32_t d, size_t lo) {
+        size_t hi = cand.size();
         while (lo < hi) {
             const size_t mid = (lo + hi + 1) / 2;
-            if (fits(mid)) lo = mid; else hi = mid - 1;
+            if (fits(d, mid)) lo = mid; else hi = mid - 1;
         }
-        fits(lo);
+        return lo;
+    };
+    int best = -1;
+    for (uint32_t d = 0; d <= maxd; d++)
+        if (compact_bytes_for(t, d, nullptr, nullptr, nullptr) <= budget) best = (int)d;
+    size_t best_k = 0;
+    if (best >= 0) {
+        candidates((uint32_t)best);
+        best_k = widest((uint32_t)best, 0);
+    } else {
+        uint32_t best_nd = 0;
+        for (uint32_t d = 0; d <= std::min<uint32_t>(maxd, 6); d++) {
+            candidates(d);
+            size_t k0 = SIZE_MAX;  // the first fitting k on a doubling grid
+            for (size_t k = 1; k <= cand.size(); k = k * 2) {
+                if (fits(d, k)) { k0 = k; break; }
+                if (k * 2 > cand.size() && k != cand.size() && fits(d, cand.size())) { k0 = cand.size(); break; }
+            }
+            if (k0 == SIZE_MAX) continue;
+            const size_t k = widest(d, k0);
+            fits(d, k);
+            if (nd_try > best_nd) best_nd = nd_try, best = (int)d, best_k = k;
+        }
+        if (best < 0) return false;
+        candidates((uint32_t)best);
     }
+    fits((uint32_t)best, best_k);
     std::vector<uint8_t> dense;
     uint32_t nd = 0;
     const size_t total = compact_bytes_for(t, (uint32_t)best, &seed, &dense, &nd);

@@ -20,7 +20,9 @@ const StagedConfig &staged_variant(int v) { return kVariants[v - 1]; }
 size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt) {
     const size_t ring = (size_t)cfg.warps * cfg.stages * 32 * cfg.k * cfg.width;
     const size_t bars = ((size_t)cfg.warps * cfg.stages * 8 + 15) / 16 * 16;
-    return 1024 + ring + bars + 256 + smem_stt;
+    // swizzled tiles (W >= 32) align the ring to the 1024-B swizzle atom at run time
+    const size_t align = cfg.swizzle && cfg.width >= 32 ? 1024 : 0;
+    return align + ring + bars + 256 + smem_stt;
 }
 
 cudaError_t launch_scan_global(int mode, uint32_t eb, uint32_t tier, const uint8_t *text, uint64_t n_total,

@@ -197,7 +197,9 @@ def test_compact_encoding_equals_dense(which):
         oidx = x - (nd - od)
         payload, count = ot[oidx].tolist()
         assert count == len(outs) and payload == (outs[0] if count == 1 else int(t.out_off[s]))
-    assert d["compact_bytes"] <= 232448 - (1024 + 32 * 2 * 512 + 512 + 256) - 1024
+    # fits next to the lean staged variant's ring (32 warps x 2 slots x 512 B, unswizzled:
+    # no alignment pad), its mbarriers, the class map and 128 B of slack
+    assert d["compact_bytes"] <= 232448 - (32 * 2 * 512 + 512 + 256) - 128
     if which == "c2":
         assert S > 15000 and d["stt_bytes"] > 1_000_000  # the dense table would not fit
 
