@@ -159,7 +159,9 @@ typedef struct {
                               scratch slot during the single emitting pass
                               (0 = auto from cap); chains with more are
                               re-scanned straight into place                 */
-    uint32_t two_pass;     /* list mode: 0 = single emitting pass (chain
+    uint32_t two_pass;     /* list mode: 0 = auto: single emitting pass, or
+                              the two passes when cap / chains > ~1K records
+                              (several matches per byte); single pass: chain
                               offsets computed inside the staged scan when
                               the text pointer is 16-byte aligned, else by
                               a separate offset scan); 1 = count pass + emit

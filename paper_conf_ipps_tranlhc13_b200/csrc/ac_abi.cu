@@ -45,6 +45,7 @@ static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slot
 // chains of >= 256 B; the global kernel's shorter chains win (C1: 1 MiB list
 // 0.037 ms global vs 0.052 ms staged).
 static const uint64_t kStagedMinBytes = 32ull << 20;
+static const uint64_t kMaxSlots = 4096;  // scratch records per chain in the single emitting pass
 static const uint64_t kStagedMinChain = 256;
 
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda).
@@ -379,7 +380,15 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         return scan(MODE_COUNT_TOTAL, "k_scan_global(count)", "k_scan_staged(count)");
     }
     // --- list mode workspace: counts | chain_end | list | tile_state | counters
-    const bool two_pass = opts && opts->two_pass == 1;
+    // Two passes (count, offsets, emit in place) when the capacity says the
+    // chains will not fit their scratch slots (> kMaxSlots records each, i.e.
+    // several matches per byte): every chain would overflow into k_rewalk.
+    // Measured (C5 English, 256 MiB): 20K patterns 13.6 -> 5.9 ms, 50K 70 ->
+    // 12 ms; the single pass stays better up to ~1K records per chain (C2:
+    // 111, 0.51 vs 0.78 ms; 5K patterns: 930, 2.96 vs 3.10 ms).
+    const bool dense_out =
+        (!opts || (opts->two_pass == 0 && opts->scratch_slots == 0)) && 4 * (cap / n_chains) + 64 > kMaxSlots;
+    const bool two_pass = (opts && opts->two_pass == 1) || dense_out;
     // in-kernel offsets: the staged kernel places its chains (decoupled
     // look-back per CTA) when the main region starts the list and the tail
     // is short; k_gather places the tail.  two_pass = 2 forces k_offsets.
@@ -417,7 +426,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     so.chain_end = chain_end;
     // single pass: each chain keeps its first q records in a scratch slot
     uint64_t q = opts && opts->scratch_slots ? opts->scratch_slots : 4 * (cap / n_chains) + 64;
-    if (q > 4096) q = 4096;
+    if (q > kMaxSlots) q = kMaxSlots;
     const uint64_t max_scratch = 8ull << 30;
     if (n_chains * q * 8 > max_scratch) q = max_scratch / (n_chains * 8);
     if (q == 0) q = 1;
