@@ -36,7 +36,12 @@ def oracle_keys(o: Oracle, text, lo=None, hi=None) -> np.ndarray:
 
 
 def gpu_keys(stt, text_np: np.ndarray, **kw) -> np.ndarray:
-    t = torch.from_numpy(np.ascontiguousarray(text_np)).cuda() if text_np.size else torch.empty(0, dtype=torch.uint8, device="cuda")
+    if not text_np.size:
+        t = torch.empty(0, dtype=torch.uint8, device="cuda")
+    else:
+        # read-only views (np.frombuffer) are copied: torch.from_numpy wants a writable array
+        a = text_np if text_np.flags.writeable and text_np.flags.c_contiguous else np.array(text_np, order="C")
+        t = torch.from_numpy(a).cuda()
     c, recs = ac.match(stt, t, **kw)
     cnt = ac.count(stt, t, **{k: v for k, v in kw.items() if k in ("kernel", "chain_bytes", "variant")})
     if c:  # the two-pass list mode and a forced-overflow single pass agree bit for bit
