@@ -304,22 +304,71 @@ uint64_t oracle_match_chunked(const ac_oracle *m, const uint8_t *text, uint64_t 
     return count;
 }
 
-/* Canonical order (reading R3): start ascending, then pattern id ascending. */
-static const uint32_t *g_sort_lens;
-typedef struct { uint64_t end; uint32_t pid; } occ_t;
+/* Canonical order (reading R3): start ascending, then pattern id ascending.
+ * Each element carries its own start, so the comparator needs no shared state
+ * and concurrent calls from several threads are safe. */
+typedef struct { uint64_t start; uint64_t end; uint32_t pid; } occ_t;
 static int cmp_occ(const void *x, const void *y) {
     const occ_t *a = (const occ_t *)x, *b = (const occ_t *)y;
-    uint64_t sa = a->end + 1 - g_sort_lens[a->pid], sb = b->end + 1 - g_sort_lens[b->pid];
-    if (sa != sb) return sa < sb ? -1 : 1;
+    if (a->start != b->start) return a->start < b->start ? -1 : 1;
     return (a->pid > b->pid) - (a->pid < b->pid);
 }
 int oracle_canonical_sort(const ac_oracle *m, uint64_t *ends, uint32_t *pids, uint64_t count) {
     occ_t *v = (occ_t *)malloc((count ? count : 1) * sizeof(occ_t));
     if (!v) return -1;
-    for (uint64_t i = 0; i < count; i++) { v[i].end = ends[i]; v[i].pid = pids[i]; }
-    g_sort_lens = m->lens;
+    for (uint64_t i = 0; i < count; i++) {
+        v[i].end = ends[i];
+        v[i].pid = pids[i];
+        v[i].start = ends[i] + 1 - m->lens[pids[i]];
+    }
     qsort(v, count, sizeof(occ_t), cmp_occ);
     for (uint64_t i = 0; i < count; i++) { ends[i] = v[i].end; pids[i] = v[i].pid; }
     free(v);
     return 0;
+}
+
+/*
+ * Multiset digest of the occurrences whose start lies in [lo, own_hi) (the
+ * window of oracle_match_window, same walk), for texts whose full list is too
+ * large to keep (SURVEY 8(c) "GPU parity": count, sum and xor of
+ * splitmix64(key) over the occurrences, order independent).  key = start *
+ * 2^24 + pid with start = base + end - len + 1 (the canonical (start, pid)
+ * pair of reading R3 written as one integer; "at the end of position").
+ * splitmix64 is the public constant-exact mixer (Steele, Lea, Flood 2014),
+ * written out here on its own.  out[0] = count, out[1] = sum mod 2^64,
+ * out[2] = xor.
+ */
+static uint64_t mix64(uint64_t x) {
+    uint64_t z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+void oracle_digest_window(const ac_oracle *m, const uint8_t *text, uint64_t n, uint64_t lo, uint64_t own_hi,
+                          uint64_t base, uint64_t *out) {
+    uint64_t halo = m->maxlen ? m->maxlen - 1 : 0;
+    uint64_t count = 0, sum = 0, x = 0;
+    if (own_hi > n) own_hi = n;
+    if (lo < own_hi) {
+        uint64_t hi = own_hi + halo < n ? own_hi + halo : n;
+        uint32_t state = 0;
+        for (uint64_t i = lo; i < hi; i++) { /* the walk of P:55-58, as walk() above */
+            uint8_t a = text[i];
+            while (oracle_goto(m, state, a) == FAIL) state = m->nodes[state].fail;
+            state = (uint32_t)oracle_goto(m, state, a);
+            const node_t *nd = &m->nodes[state];
+            for (uint32_t k = 0; k < nd->n_out; k++) {
+                uint32_t p = nd->out[k];
+                uint64_t start = i + 1 - m->lens[p];
+                if (start >= own_hi) continue;
+                uint64_t h = mix64(((base + start) << 24) | p);
+                count++;
+                sum += h;
+                x ^= h;
+            }
+        }
+    }
+    out[0] = count;
+    out[1] = sum;
+    out[2] = x;
 }

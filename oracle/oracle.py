@@ -14,6 +14,7 @@ from __future__ import annotations
 import ctypes
 import os
 import subprocess
+from concurrent.futures import ThreadPoolExecutor
 from pathlib import Path
 
 import numpy as np
@@ -69,6 +70,9 @@ def _load():
         lib.oracle_match_chunked.restype = ctypes.c_uint64
         lib.oracle_match_chunked.argtypes = [ctypes.c_void_p, _u8p, ctypes.c_uint64, ctypes.c_uint64,
                                              ctypes.c_uint64, _u64p, _u32p, ctypes.c_uint64]
+        lib.oracle_digest_window.restype = None
+        lib.oracle_digest_window.argtypes = [ctypes.c_void_p, _u8p, ctypes.c_uint64, ctypes.c_uint64,
+                                             ctypes.c_uint64, ctypes.c_uint64, _u64p]
         lib.oracle_canonical_sort.restype = ctypes.c_int
         lib.oracle_canonical_sort.argtypes = [ctypes.c_void_p, _u64p, _u32p, ctypes.c_uint64]
         _lib = lib
@@ -182,3 +186,50 @@ class Oracle:
             rc = self._lib.oracle_canonical_sort(self._h, _ptr(ends, _u64p), _ptr(pids, _u32p), ends.size)
             if rc != 0:
                 raise MemoryError("oracle_canonical_sort")
+
+    # --- whole texts on every host core --------------------------------------
+    # The chunked mode of P:163-164 one level up: window [lo, hi) is walked
+    # from state 0 over [lo, min(hi + maxlen - 1, n)) and keeps the
+    # occurrences whose start it owns (reading R9), one window per thread.
+    # ctypes releases the GIL for the duration of each C call, so the windows
+    # run concurrently.  Concatenating the windows' canonical lists in window
+    # order is the canonical list of the whole text (start-major order).
+    def _windows(self, n: int, threads: int | None, min_window: int = 1 << 20):
+        threads = threads or os.cpu_count() or 1
+        k = max(1, min(4 * threads, (n + min_window - 1) // min_window))
+        cuts = [n * i // k for i in range(k + 1)]
+        return threads, [(cuts[i], cuts[i + 1]) for i in range(k) if cuts[i] < cuts[i + 1]]
+
+    def match_parallel(self, text, threads: int | None = None, base: int = 0):
+        """(ends, pids) of the whole text in canonical order, windows on `threads` cores."""
+        t = _as_u8(text)
+        threads, wins = self._windows(t.size, threads)
+
+        def one(w):
+            return self.match_window(t, w[0], w[1], base=base, canonical=True)
+
+        with ThreadPoolExecutor(threads) as ex:
+            parts = list(ex.map(one, wins))
+        if not parts:
+            return np.zeros(0, np.uint64), np.zeros(0, np.uint32)
+        return np.concatenate([p[0] for p in parts]), np.concatenate([p[1] for p in parts])
+
+    def digest_window(self, text, lo: int, own_hi: int, base: int = 0):
+        """(count, sum, xor) of splitmix64(start << 24 | pid) over the window's owned occurrences."""
+        t = _as_u8(text)
+        out = np.zeros(3, dtype=np.uint64)
+        self._lib.oracle_digest_window(self._h, _ptr(t, _u8p), t.size, lo, own_hi, base, _ptr(out, _u64p))
+        return int(out[0]), int(out[1]), int(out[2])
+
+    def digest_parallel(self, text, threads: int | None = None, base: int = 0):
+        """Multiset digest of the whole text: (count, sum mod 2^64, xor)."""
+        t = _as_u8(text)
+        threads, wins = self._windows(t.size, threads)
+        with ThreadPoolExecutor(threads) as ex:
+            parts = list(ex.map(lambda w: self.digest_window(t, w[0], w[1], base=base), wins))
+        c, sm, x = 0, 0, 0
+        for pc, ps, px in parts:
+            c += pc
+            sm = (sm + ps) & ((1 << 64) - 1)
+            x ^= px
+        return c, sm, x

@@ -124,6 +124,7 @@ def test_functions_match_their_definitions(seed):
     assert set(strs.values()) == prefixes and len(strs) == o.num_states
     by_str = {v: k for k, v in strs.items()}
     for s, w in strs.items():
+        assert o.depth(s) == len(w)  # depth = length of the state's string (trie level)
         if s:
             suf = next(w[i:] for i in range(1, len(w) + 1) if w[i:] in prefixes)
             assert o.fail(s) == by_str[suf]
@@ -282,3 +283,86 @@ def test_all_byte_values():
     pats = [bytes([b]) for b in range(256)] + [text[100:104], text[4000:4010], b"\x00\x00"]
     o = Oracle(pats)
     assert _pairs(*o.match(text)) == brute_matches(text, pats)
+
+
+# ---------------------------------------------------------------------------
+# Whole-text runners used by the full-size GPU parity tests: the parallel
+# window runner and the multiset digest, pinned to brute force
+# ---------------------------------------------------------------------------
+_M64 = (1 << 64) - 1
+
+
+def _mix64(x: int) -> int:
+    """splitmix64 (Steele, Lea, Flood 2014), written out independently."""
+    z = (x + 0x9E3779B97F4A7C15) & _M64
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & _M64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & _M64
+    return z ^ (z >> 31)
+
+
+def test_mix64_known_values():
+    # splitmix64 stream seeded with 0: the published first outputs
+    assert _mix64(0) == 0xE220A8397B1DCDAF
+    assert _mix64(0x9E3779B97F4A7C15) == 0x6E789E6AA1B965F4
+
+
+@pytest.mark.parametrize("seed", range(200))
+def test_digest_window_against_brute_force(seed):
+    rng = random.Random(7000 + seed)
+    A = rng.randint(1, 4)
+    alphabet = list(range(97, 97 + A))
+    pats = [bytes(rng.choice(alphabet) for _ in range(rng.randint(1, 6))) for _ in range(rng.randint(1, 8))]
+    text = bytes(rng.choice(alphabet) for _ in range(rng.randint(0, 200)))
+    lo = rng.randint(0, len(text))
+    hi = rng.randint(lo, len(text) + 3)
+    base = rng.choice([0, 1, 12345, 1 << 33])
+    o = Oracle(pats)
+    want = [(e - len(pats[p]) + 1, p) for e, p in brute_matches(text, pats)]
+    want = [(st, p) for st, p in want if lo <= st < min(hi, len(text))]
+    hs = [_mix64(((base + st) << 24) | p) for st, p in want]
+    sm, x = 0, 0
+    for h in hs:
+        sm = (sm + h) & _M64
+        x ^= h
+    assert o.digest_window(text, lo, hi, base=base) == (len(want), sm, x)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_parallel_runners_against_brute_force(seed):
+    rng = random.Random(9100 + seed)
+    A = rng.randint(1, 3)
+    alphabet = list(range(97, 97 + A))
+    pats = [bytes(rng.choice(alphabet) for _ in range(rng.randint(1, 7))) for _ in range(rng.randint(1, 10))]
+    text = bytes(rng.choice(alphabet) for _ in range(rng.randint(0, 3000)))
+    o = Oracle(pats)
+    # tiny windows so the 3000-byte text is split many times across threads
+    o._windows = lambda n, threads, min_window=37: Oracle._windows(o, n, 5, min_window)
+    want = brute_matches(text, pats)
+    ends, pids = o.match_parallel(text)
+    assert _pairs(ends, pids) == want
+    hs = [_mix64(((e - len(pats[p]) + 1) << 24) | p) for e, p in want]
+    sm, x = 0, 0
+    for h in hs:
+        sm = (sm + h) & _M64
+        x ^= h
+    assert o.digest_parallel(text) == (len(want), sm, x)
+
+
+def test_canonical_sort_is_reentrant():
+    # many threads sorting different dictionaries' lists at once must each
+    # get their own canonical order (the comparator keeps no shared state)
+    from concurrent.futures import ThreadPoolExecutor
+    cases = []
+    for seed in range(16):
+        rng = random.Random(seed)
+        pats = [bytes(rng.choice(b"ab") for _ in range(rng.randint(1, 9))) for _ in range(6)]
+        text = bytes(rng.choice(b"ab") for _ in range(20000))
+        cases.append((Oracle(pats), text, brute_matches(text, pats)))
+
+    def run(c):
+        o, text, want = c
+        ends, pids = o.match(text)
+        return _pairs(ends, pids) == want
+
+    with ThreadPoolExecutor(8) as ex:
+        assert all(ex.map(run, cases * 2))
