@@ -79,9 +79,21 @@ typedef struct ac_table ac_table;
  * prefix in shared memory, the rest through L1/L2.  GLOBAL: L1/L2 only.
  * COMPACT: dense rows for shallow states + 8-byte default-transition records
  * for the others + an output table, all in shared memory (<= 32768 states,
- * <= 127 classes).  AUTO = SMEM if the dense table
- * fits, else COMPACT if that fits, else GLOBAL. */
-enum { AC_TIER_AUTO = 0, AC_TIER_SMEM = 1, AC_TIER_HYBRID = 2, AC_TIER_GLOBAL = 3, AC_TIER_COMPACT = 4 };
+ * <= 127 classes).  SPLIT: the hot BFS part of a
+ * large automaton in shared memory -- dense 16-bit rows for the shallow
+ * levels, 8-byte default-transition records for the next states -- and the
+ * full 32-bit table in global memory (L1/L2) for the cold states (DESIGN.md
+ * "SPLIT tier"; SURVEY 8(a)-a5 tier (ii)).  AUTO = SMEM if the dense table
+ * fits, else COMPACT if that fits, else GLOBAL with the two-byte walk for
+ * <= 8 classes, else SPLIT. */
+enum {
+    AC_TIER_AUTO = 0,
+    AC_TIER_SMEM = 1,
+    AC_TIER_HYBRID = 2,
+    AC_TIER_GLOBAL = 3,
+    AC_TIER_COMPACT = 4,
+    AC_TIER_SPLIT = 5
+};
 
 typedef struct {
     uint32_t struct_size;  /* sizeof(ac_build_opts)                          */
@@ -135,6 +147,13 @@ typedef struct {
     uint32_t stride;       /* 1 or 2 (two-byte table present)                */
     uint32_t stride2_cols; /* row stride of the two-byte table (C*C, odd)   */
     uint64_t stt2_bytes;
+    /* SPLIT tier (valid when split_bytes != 0): BFS ids [0, split_dense) are
+     * dense rows of split_dstride u16 entries, ids [split_dense, split_dense +
+     * split_records) are 8-byte records {lo32 = fd | c1 << 16 | c2 << 24,
+     * hi32 = t1 | t2 << 16}; a u16 entry is 2 x + flag, or 0xFFFF = read the
+     * global table; split_cold_records of the records are cold (fd 0xFFFF). */
+    uint32_t split_dense, split_records, split_dstride, split_cold_records;
+    uint64_t split_bytes;
 } ac_stt_info;
 
 /* Scan variants (SURVEY 8(f) NEXT-1 ablations are selectable here). */
@@ -200,7 +219,10 @@ ac_status ac_stt_pattern_lengths(const ac_stt *stt, uint32_t *lens);
 
 /* ---------------------------------------------------------------- phase 2
  * ac_match: scans d_text[0, n) (DEVICE memory, any alignment, n may be 0)
- * and reports every occurrence.
+ * and reports every occurrence.  The list is produced in one emitting pass
+ * when cap <= n (at most one record per text byte of room), else in two
+ * (count, then emit in place) -- cap is read as the caller's density bound,
+ * no count pass is run to plan.
  *   d_out == NULL : count only; *count = number of occurrences.
  *   d_out != NULL : DEVICE buffer of `cap` records; on AC_OK it holds the
  *                   *count records in canonical order.  If the count exceeds
@@ -245,6 +267,10 @@ ac_status ac_match_segments(const ac_stt *stt, const uint8_t *d_text, const uint
  * and the name of launch i (NULL if out of range). */
 uint32_t ac_last_launch_count(void);
 const char *ac_last_launch_name(uint32_t i);
+/* Owned text bytes scan launch i walked (0 for non-scan launches: offsets,
+ * gather, re-walk).  For per-kernel throughput accounting; halo re-walks are
+ * not counted (reading R14). */
+uint64_t ac_last_launch_text_bytes(uint32_t i);
 /* Bytes per scratch record of the last list-mode ac_match_async on this
  * thread: 4 (narrow: offset in chain and pattern id share 32 bits), 8, or 0
  * (count mode / two-pass mode: no scratch).  For traffic accounting. */
@@ -280,6 +306,9 @@ ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm)
  * stride2_cols u32, column c1*C + c2 -> delta(delta(s,c1),c2) | bit 31 =
  * output(final) != {} | bit 30 = output(middle) != {}. */
 ac_status ac_table_export_stride2(const ac_table *t, uint32_t *tab);
+/* opts->tier == AC_TIER_SPLIT (ac_compile) builds the SPLIT shared-memory
+ * part for the default budget (32-bit table); copies its split_bytes. */
+ac_status ac_table_export_split(const ac_table *t, void *blob);
 void ac_table_free(ac_table *t);
 
 /* ------------------------------------------------------------ diagnostics */

@@ -27,14 +27,14 @@ LIB_PATH = _PKG / "libac.so"
 
 AC_OK, AC_ERR_INVALID_ARG, AC_ERR_EMPTY_PATTERN, AC_ERR_TOO_LARGE = 0, 1, 2, 3
 AC_ERR_CAPACITY, AC_ERR_NO_MEMORY, AC_ERR_CUDA, AC_ERR_NO_DEVICE = 4, 5, 6, 7
-TIER_AUTO, TIER_SMEM, TIER_HYBRID, TIER_GLOBAL, TIER_COMPACT = 0, 1, 2, 3, 4
+TIER_AUTO, TIER_SMEM, TIER_HYBRID, TIER_GLOBAL, TIER_COMPACT, TIER_SPLIT = 0, 1, 2, 3, 4, 5
 KERNEL_AUTO, KERNEL_STAGED, KERNEL_GLOBAL = 0, 1, 2
-TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global", 4: "compact"}
+TIER_NAMES = {1: "smem", 2: "hybrid", 3: "global", 4: "compact", 5: "split"}
 
 EXPORTED = [
     "ac_build", "ac_free", "ac_stt_query", "ac_stt_pattern_lengths", "ac_match", "ac_match_shard",
-    "ac_match_async", "ac_match_segments", "ac_last_launch_count", "ac_last_launch_name", "ac_last_scratch_record_bytes", "ac_match_host", "ac_compile", "ac_table_query",
-    "ac_table_export", "ac_table_export_compact", "ac_table_export_stride2", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
+    "ac_match_async", "ac_match_segments", "ac_last_launch_count", "ac_last_launch_name", "ac_last_launch_text_bytes", "ac_last_scratch_record_bytes", "ac_match_host", "ac_compile", "ac_table_query",
+    "ac_table_export", "ac_table_export_compact", "ac_table_export_stride2", "ac_table_export_split", "ac_table_free", "ac_status_string", "ac_last_error", "ac_version",
 ]
 
 
@@ -63,7 +63,10 @@ class ac_stt_info(ctypes.Structure):
                 ("compact_dense", ctypes.c_uint32), ("compact_od", ctypes.c_uint32), ("compact_os", ctypes.c_uint32),
                 ("compact_dstride", ctypes.c_uint32), ("compact_sparse_off", ctypes.c_uint32),
                 ("compact_out_off", ctypes.c_uint32), ("compact_bytes", ctypes.c_uint64),
-                ("stride", ctypes.c_uint32), ("stride2_cols", ctypes.c_uint32), ("stt2_bytes", ctypes.c_uint64)]
+                ("stride", ctypes.c_uint32), ("stride2_cols", ctypes.c_uint32), ("stt2_bytes", ctypes.c_uint64),
+                ("split_dense", ctypes.c_uint32), ("split_records", ctypes.c_uint32),
+                ("split_dstride", ctypes.c_uint32), ("split_cold_records", ctypes.c_uint32),
+                ("split_bytes", ctypes.c_uint64)]
 
 
 class ac_match_opts(ctypes.Structure):
@@ -97,6 +100,7 @@ def lib():
         L.ac_table_export.argtypes = [_vp, _vp, _vp, _vp, _vp]
         L.ac_table_export_compact.argtypes = [_vp, _vp, _vp]
         L.ac_table_export_stride2.argtypes = [_vp, _vp]
+        L.ac_table_export_split.argtypes = [_vp, _vp]
         L.ac_stt_pattern_lengths.argtypes = [_vp, _vp]
         L.ac_match.argtypes = [_vp, _vp, _u64, _vp, _u64, _u64p, _vp]
         L.ac_match_shard.argtypes = [_vp, _vp, _u64, _u64, _u64, _vp, _u64, _u64p, _vp]
@@ -107,6 +111,8 @@ def lib():
         L.ac_last_launch_count.argtypes = []
         L.ac_last_launch_name.restype = ctypes.c_char_p
         L.ac_last_launch_name.argtypes = [_u32]
+        L.ac_last_launch_text_bytes.restype = _u64
+        L.ac_last_launch_text_bytes.argtypes = [_u32]
         L.ac_last_scratch_record_bytes.restype = _u32
         L.ac_last_scratch_record_bytes.argtypes = []
         L.ac_status_string.restype = ctypes.c_char_p
@@ -320,6 +326,12 @@ def last_launch_names() -> list[str]:
     return [L.ac_last_launch_name(i).decode() for i in range(L.ac_last_launch_count())]
 
 
+def last_launch_text_bytes() -> list[int]:
+    """Owned text bytes each launch of the last match_async walked (0 = not a scan)."""
+    L = lib()
+    return [int(L.ac_last_launch_text_bytes(i)) for i in range(min(16, int(L.ac_last_launch_count())))]
+
+
 def last_scratch_record_bytes() -> int:
     """4 (narrow), 8 or 0: scratch bytes per record of the last list-mode call."""
     return int(lib().ac_last_scratch_record_bytes())
@@ -354,16 +366,18 @@ class HostTable:
     compact: "object" = None   # COMPACT blob (uint8) if requested
     stt2: "object" = None      # two-byte table (uint32, S x stride2_cols) if requested
     perm: "object" = None      # compact id -> dense BFS id
+    split: "object" = None     # SPLIT shared-memory part (uint8) if requested
 
 
 def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact: bool = False,
-                  stride: int = 0) -> HostTable:
+                  stride: int = 0, split: bool = False) -> HostTable:
     """Phase 1 on the host only (no device) -- for builder tests."""
     import numpy as np
     L = lib()
     pats, bufs, ptrs, lens = _pattern_arrays(patterns)
     h = ctypes.c_void_p()
-    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=TIER_COMPACT if compact else TIER_AUTO, stride=stride)
+    tier = TIER_COMPACT if compact else TIER_SPLIT if split else TIER_AUTO
+    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=tier, stride=stride)
     _check(L.ac_compile(ptrs, lens, len(pats), ctypes.byref(o), ctypes.byref(h)))
     try:
         info = ac_stt_info()
@@ -385,7 +399,11 @@ def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact
             t2 = np.zeros(d["n_states"] * d["stride2_cols"], dtype=np.uint32)
             _check(L.ac_table_export_stride2(h, t2.ctypes.data))
             t2 = t2.reshape(d["n_states"], d["stride2_cols"])
+        sp = None
+        if split:
+            sp = np.zeros(d["split_bytes"], dtype=np.uint8)
+            _check(L.ac_table_export_split(h, sp.ctypes.data))
         return HostTable(d, cm, stt.reshape(d["n_states"], d["row_stride"]), off, ids[:d["out_entries"]],
-                         compact=blob, stt2=t2, perm=perm)
+                         compact=blob, stt2=t2, perm=perm, split=sp)
     finally:
         L.ac_table_free(h)

@@ -21,6 +21,7 @@ static thread_local std::string g_err;
 static thread_local uint32_t g_launches = 0;
 static thread_local uint32_t g_scratch_rec = 0;  // bytes per scratch record of the last list-mode call
 static thread_local const char *g_names[16];
+static thread_local uint64_t g_bytes[16];  // text bytes each scan launch walks (owned + halo), 0 otherwise
 
 void set_error(const std::string &msg) { g_err = msg; }
 
@@ -103,17 +104,39 @@ static ac_status side_stream(int device, SideStream **out) {
     return AC_OK;
 }
 
-static void keep_pool(int device) {
+// libac's own stream-ordered memory pool per device: workspace and scratch
+// are reused from call to call (a list-mode call allocates ~GBs of scratch)
+// without touching the device's default pool, which the host application's
+// allocator may rely on; memory above the release threshold goes back to the
+// device at the next synchronisation.
+static const uint64_t kPoolKeepBytes = 16ull << 30;
+static cudaMemPool_t lib_pool(int device) {
     static std::mutex mu;
-    static bool done[64] = {false};
+    static cudaMemPool_t pools[64] = {};
+    if (device < 0 || device >= 64) return nullptr;
     std::lock_guard<std::mutex> lk(mu);
-    if (device < 0 || device >= 64 || done[device]) return;
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
-        uint64_t thr = UINT64_MAX;
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    if (!pools[device]) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = device;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        uint64_t thr = kPoolKeepBytes;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[device] = p;
     }
-    done[device] = true;
+    return pools[device];
+}
+
+// Stream-ordered allocation from libac's pool (the default pool if the
+// private one could not be created); freed with cudaFreeAsync.
+static cudaError_t ws_alloc(void **p, size_t bytes, cudaStream_t s, int device) {
+    cudaMemPool_t pool = lib_pool(device);
+    return pool ? cudaMallocFromPoolAsync(p, bytes, pool, s) : cudaMallocAsync(p, bytes, s);
 }
 
 static ac_status check_device(int device, cudaDeviceProp *prop) {
@@ -170,6 +193,23 @@ static SttView view_of(const ac_stt *h, int v) {
     s.stt2 = v ? h->d_stt2 : nullptr;  // only the staged kernel walks two bytes per lookup
     s.stride2 = h->host.stride2;
     s.n_classes = h->host.n_classes;
+    s.sblob = nullptr;
+    s.s_dense = s.s_rec = s.s_row_bytes = s.s_rec_x0 = 0;
+    if (h->tier == AC_TIER_SPLIT) {
+        // the staged kernel stages the split blob; the global-only kernel
+        // (head/tail chains, short texts, re-walks) reads the global table
+        s.smem_rows = 0;
+        s.smem_bytes = 0;
+        if (v && h->host.split.size() <= stt_budget(h, v)) {
+            s.sblob = h->d_split;
+            s.smem_bytes = (uint32_t)h->host.split.size();
+            s.s_dense = h->host.s_dense;
+            s.s_rec = h->host.s_rec;
+            s.s_row_bytes = 2 * h->host.s_dstride;
+            s.s_rec_x0 = s.s_dense * s.s_row_bytes - 8u * s.s_dense;
+        }
+        return s;
+    }
     if (h->tier == AC_TIER_COMPACT) {
         s.smem_rows = h->host.n_states;
         s.smem_bytes = (uint32_t)h->host.compact.size();
@@ -187,6 +227,7 @@ static size_t smem_of(const ac_stt *, const SttView &v) { return ((size_t)v.smem
 // The kernel's tier: SMEM only when every row is resident, GLOBAL when none.
 static uint32_t tier_of(const ac_stt *h, const SttView &v) {
     if (h->tier == AC_TIER_COMPACT) return AC_TIER_COMPACT;
+    if (h->tier == AC_TIER_SPLIT) return v.sblob ? AC_TIER_SPLIT : AC_TIER_GLOBAL;
     if (v.smem_rows == 0) return AC_TIER_GLOBAL;
     if (v.smem_rows >= h->host.n_states) return AC_TIER_SMEM;
     return AC_TIER_HYBRID;
@@ -196,6 +237,8 @@ static void free_device(ac_stt *h) {
     cudaFree(h->d_stt);
     cudaFree(h->d_stt2);
     h->d_stt2 = nullptr;
+    cudaFree(h->d_split);
+    h->d_split = nullptr;
     cudaFree(h->d_class_map);
     cudaFree(h->d_out_off);
     cudaFree(h->d_out_ids);
@@ -232,12 +275,16 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     const bool emit = d_out != nullptr;
     void **ev = opts ? opts->events : nullptr;
     const uint32_t nev = opts ? opts->n_events : 0;
-    auto pre = [&]() {
-        if (ev && g_launches < nev) cudaEventRecord(static_cast<cudaEvent_t>(ev[2 * g_launches]), stream);
+    // per-launch timing events go on the stream the kernel runs on
+    auto pre = [&](cudaStream_t on) {
+        if (ev && g_launches < nev) cudaEventRecord(static_cast<cudaEvent_t>(ev[2 * g_launches]), on);
     };
-    auto post = [&](const char *name) {
-        if (ev && g_launches < nev) cudaEventRecord(static_cast<cudaEvent_t>(ev[2 * g_launches + 1]), stream);
-        if (g_launches < 16) g_names[g_launches] = name;
+    auto post = [&](const char *name, cudaStream_t on, uint64_t text_bytes) {
+        if (ev && g_launches < nev) cudaEventRecord(static_cast<cudaEvent_t>(ev[2 * g_launches + 1]), on);
+        if (g_launches < 16) {
+            g_names[g_launches] = name;
+            g_bytes[g_launches] = text_bytes;
+        }
         g_launches++;
     };
     AC_CUDA(cudaMemsetAsync(d_res, 0, sizeof(ac_result), stream), "memset result");
@@ -256,6 +303,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     if (variant == 0) {
         variant = kAutoVariant;
         if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
+        if (h->tier == AC_TIER_SPLIT && h->host.split.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
     }
     if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, variant)) {
         set_error("staged variant " + std::to_string(variant) + " has no room for the COMPACT table");
@@ -297,7 +345,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             g.n_chains = n_main;
             g.chain0 = ra.n_chains;
             g.n_readable = n_total - head;
-            g.text_evict_first = (tier_s == AC_TIER_GLOBAL || tier_s == AC_TIER_HYBRID) ? 1u : 0u;
+            g.text_evict_first =
+                (tier_s == AC_TIER_GLOBAL || tier_s == AC_TIER_HYBRID || tier_s == AC_TIER_SPLIT) ? 1u : 0u;
             PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
             if (!enc) {
                 set_error("cuTensorMapEncodeTiled unavailable from the driver");
@@ -359,18 +408,18 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
                 AC_CUDA(cudaStreamWaitEvent(side->stream, side->fork, 0), "cudaStreamWaitEvent(fork)");
                 gs = side->stream;
             }
-            pre();
+            pre(gs);
             AC_CUDA(launch_scan_global(mode, eb, tier_g, d_text, n_total, sg, ra, rb, so, smem_g, gs), gname);
-            post(gname);
+            post(gname, gs, (ra.hi - ra.lo) + (rb.hi - rb.lo));
             if (side) AC_CUDA(cudaEventRecord(side->join, side->stream), "cudaEventRecord(join)");
         }
         if (g.n_chains) {
-            pre();
+            pre(stream);
             ScanOut sso = so;
             if (mode == MODE_EMIT_OPT) sso.nbits = nm_bits;
             AC_CUDA(launch_scan_staged(mode, eb, tier_s, variant, tmap, d_text + g.m0, ss, g, sso, smem_s, stream),
                     sname);
-            post(sname);
+            post(sname, stream, g.n_chains * g.chain_len);
         }
         if (side) AC_CUDA(cudaStreamWaitEvent(stream, side->join, 0), "cudaStreamWaitEvent(join)");
         return AC_OK;
@@ -380,15 +429,32 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         return scan(MODE_COUNT_TOTAL, "k_scan_global(count)", "k_scan_staged(count)");
     }
     // --- list mode workspace: counts | chain_end | list | tile_state | counters
-    // Two passes (count, offsets, emit in place) when the capacity says the
-    // chains will not fit their scratch slots (> kMaxSlots records each, i.e.
-    // several matches per byte): every chain would overflow into k_rewalk.
-    // Measured (C5 English, 256 MiB): 20K patterns 13.6 -> 5.9 ms, 50K 70 ->
-    // 12 ms; the single pass stays better up to ~1K records per chain (C2:
-    // 111, 0.51 vs 0.78 ms; 5K patterns: 930, 2.96 vs 3.10 ms).
-    const bool dense_out =
-        (!opts || (opts->two_pass == 0 && opts->scratch_slots == 0)) && 4 * (cap / n_chains) + 64 > kMaxSlots;
-    const bool two_pass = (opts && opts->two_pass == 1) || dense_out;
+    // Two passes (count, offsets, emit in place) for dense outputs (several
+    // matches per byte), where every chain would overflow its scratch slot
+    // into k_rewalk.  Measured (C5 English, 256 MiB): 20K patterns (2 per
+    // byte) 13.6 -> 5.9 ms, 50K 70 -> 12 ms; the single pass stays better up
+    // to ~1K records per chain (C2, 0.06 per byte: 0.51 vs 0.78 ms; 5K
+    // patterns, 0.5 per byte: 2.96 vs 3.10 ms).  The capacity is read as the
+    // caller's density bound: room for more than one record per owned text
+    // byte selects the two-pass emission (no count pass is needed to plan).
+    const bool dense_out = (!opts || (opts->two_pass == 0 && opts->scratch_slots == 0)) && cap > n_owned;
+    bool two_pass = (opts && opts->two_pass == 1) || dense_out;
+    // single pass: each chain keeps its first q records in a scratch slot;
+    // if the slots cannot be allocated the call falls back to two passes
+    uint64_t q = opts && opts->scratch_slots ? opts->scratch_slots : 4 * (cap / n_chains) + 64;
+    if (q > kMaxSlots) q = kMaxSlots;
+    const uint64_t max_scratch = 8ull << 30;
+    if (n_chains * q * 8 > max_scratch) q = max_scratch / (n_chains * 8);
+    if (q == 0) q = 1;
+    void *scratch = nullptr;
+    if (!two_pass) {
+        cudaError_t e = ws_alloc(&scratch, n_chains * q * 8, stream, h->device);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            scratch = nullptr;
+            two_pass = true;
+        }
+    }
     // in-kernel offsets: the staged kernel places its chains (decoupled
     // look-back per CTA) when the main region starts the list and the tail
     // is short; k_gather places the tail.  two_pass = 2 forces k_offsets.
@@ -399,7 +465,13 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     const size_t tiles = offsets_tiles(n_chains);
     const size_t bytes = n_chains * 8 * 3 + tiles * 8 + 16 + n_lb * 8;
     void *ws = nullptr;
-    AC_CUDA(cudaMallocAsync(&ws, bytes, stream), "cudaMallocAsync(workspace)");
+    {
+        cudaError_t e = ws_alloc(&ws, bytes, stream, h->device);
+        if (e != cudaSuccess) {
+            if (scratch) cudaFreeAsync(scratch, stream);
+            return cuda_fail(e, "cudaMallocAsync(workspace)");
+        }
+    }
     uint64_t *counts = static_cast<uint64_t *>(ws);
     uint64_t *chain_end = counts + n_chains;
     uint64_t *list = chain_end + n_chains;
@@ -408,6 +480,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     unsigned int *list_n = counter + 1;
     unsigned long long *lb = place ? reinterpret_cast<unsigned long long *>(counter + 4) : nullptr;
     so.tile_state = lb;
+    so.ticket = place ? counter + 2 : nullptr;
     so.chain_end_w = chain_end;
     TailPlace tp{lb, n_lb, rb.chain0, rb.n_chains, cap};
     // narrow scratch records for the staged kernel's deferred emission (one
@@ -424,19 +497,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     g_scratch_rec = two_pass ? 0u : nm.nbits ? 4u : 8u;
     so.chain_counts = counts;
     so.chain_end = chain_end;
-    // single pass: each chain keeps its first q records in a scratch slot
-    uint64_t q = opts && opts->scratch_slots ? opts->scratch_slots : 4 * (cap / n_chains) + 64;
-    if (q > kMaxSlots) q = kMaxSlots;
-    const uint64_t max_scratch = 8ull << 30;
-    if (n_chains * q * 8 > max_scratch) q = max_scratch / (n_chains * 8);
-    if (q == 0) q = 1;
-    void *scratch = nullptr;
-    if (!two_pass) {
-        cudaError_t e = cudaMallocAsync(&scratch, n_chains * q * 8, stream);
-        if (e != cudaSuccess) {
-            cudaFreeAsync(ws, stream);
-            return cuda_fail(e, "cudaMallocAsync(scratch)");
-        }
+    if (scratch) {
         so.scratch = static_cast<uint64_t *>(scratch);
         so.q = (uint32_t)q;
     }
@@ -445,30 +506,30 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         if (two_pass) {
             ac_status rc = scan(MODE_COUNT_CHAINS, "k_scan_global(count)", "k_scan_staged(count)");
             if (rc != AC_OK) return rc;
-            pre();
+            pre(stream);
             AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream),
                     "k_offsets");
-            post("k_offsets");
+            post("k_offsets", stream, 0);
             return scan(MODE_EMIT, "k_scan_global(emit)", "k_scan_staged(emit)");
         }
         ac_status rc = scan(MODE_EMIT_OPT, "k_scan_global(emit1)", "k_scan_staged(emit1)");
         if (rc != AC_OK) return rc;
         if (!place) {
-            pre();
+            pre(stream);
             AC_CUDA(launch_offsets(counts, n_chains, chain_end, tile_state, counter, d_res, cap, 1, stream),
                     "k_offsets");
-            post("k_offsets");
+            post("k_offsets", stream, 0);
         }
-        pre();
+        pre(stream);
         AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, tp, nm,
                               h->num_sms, stream),
                 "k_gather");
-        post("k_gather");
-        pre();
+        post("k_gather", stream, 0);
+        pre(stream);
         AC_CUDA(launch_rewalk(eb, tier_g, d_text, n_total, sg, ra, rb, g, so, list, list_n, smem_g, h->num_sms,
                               stream),
                 "k_rewalk");
-        post("k_rewalk");
+        post("k_rewalk", stream, 0);
         return AC_OK;
     };
     const ac_status rc = run();
@@ -495,7 +556,10 @@ static ac_status match_segments(const ac_stt *h, const uint8_t *d_text, const ui
     so.res = d_res;
     so.out = reinterpret_cast<uint64_t *>(d_out);
     auto note = [&](const char *name) {
-        if (g_launches < 16) g_names[g_launches] = name;
+        if (g_launches < 16) {
+            g_names[g_launches] = name;
+            g_bytes[g_launches] = 0;
+        }
         g_launches++;
     };
     if (!d_out) {
@@ -507,7 +571,7 @@ static ac_status match_segments(const ac_stt *h, const uint8_t *d_text, const ui
     }
     const size_t tiles = offsets_tiles(n_seg);
     void *ws = nullptr;
-    AC_CUDA(cudaMallocAsync(&ws, n_seg * 16 + tiles * 8 + 16, stream), "cudaMallocAsync(workspace)");
+    AC_CUDA(ws_alloc(&ws, n_seg * 16 + tiles * 8 + 16, stream, h->device), "cudaMallocAsync(workspace)");
     uint64_t *counts = static_cast<uint64_t *>(ws);
     uint64_t *chain_end = counts + n_seg;
     uint64_t *tile_state = chain_end + n_seg;
@@ -604,17 +668,21 @@ static ac_status match_host_pipelined(const ac_stt *stt, const uint8_t *h_text, 
     ac_match_t *d_out = nullptr;
     ac_result *d_res = nullptr;
     auto cleanup = [&]() {
+        // the copy streams still read d_out / the text buffers: drain them
+        // before the frees are enqueued (stream-ordered reuse is per stream)
+        cudaStreamSynchronize(P->d2h);
+        cudaStreamSynchronize(P->h2d);
         for (auto &b : tb)
             if (b) cudaFreeAsync(b, s);
         if (d_out) cudaFreeAsync(d_out, s);
         if (d_res) cudaFreeAsync(d_res, s);
-        cudaStreamSynchronize(P->d2h);
-        cudaStreamSynchronize(P->h2d);
         cudaStreamSynchronize(s);
     };
-    cudaError_t e = cudaMallocAsync(&d_res, nch * sizeof(ac_result), s);
-    for (int b = 0; b < 2 && e == cudaSuccess && n; b++) e = cudaMallocAsync(&tb[b], CH + H + 16, s);
-    if (e == cudaSuccess && emit) e = cudaMallocAsync(&d_out, (cap ? cap : 1) * sizeof(ac_match_t), s);
+    cudaError_t e = ws_alloc(reinterpret_cast<void **>(&d_res), nch * sizeof(ac_result), s, stt->device);
+    for (int b = 0; b < 2 && e == cudaSuccess && n; b++)
+        e = ws_alloc(reinterpret_cast<void **>(&tb[b]), CH + H + 16, s, stt->device);
+    if (e == cudaSuccess && emit)
+        e = ws_alloc(reinterpret_cast<void **>(&d_out), (cap ? cap : 1) * sizeof(ac_match_t), s, stt->device);
     // the copy streams must see the allocations
     if (e == cudaSuccess) e = cudaEventRecord(P->freed[0], s);
     if (e == cudaSuccess) e = cudaEventRecord(P->freed[1], s);
@@ -702,6 +770,7 @@ const char *ac_version(void) { return "libac 0.1 sm_100a (TMA-staged + global-on
 uint32_t ac_last_launch_count(void) { return g_launches; }
 uint32_t ac_last_scratch_record_bytes(void) { return g_scratch_rec; }
 const char *ac_last_launch_name(uint32_t i) { return i < g_launches && i < 16 ? g_names[i] : nullptr; }
+uint64_t ac_last_launch_text_bytes(uint32_t i) { return i < g_launches && i < 16 ? g_bytes[i] : 0; }
 
 ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n, const ac_build_opts *opts,
                      ac_table **out) {
@@ -718,7 +787,17 @@ ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint3
     if (!t) return AC_ERR_NO_MEMORY;
     ac_status rc;
     try {
-        rc = compile_table(patterns, lens, n, opts, *t);
+        ac_build_opts o4;
+        const bool split = opts && opts->tier == AC_TIER_SPLIT;
+        if (split) {  // the SPLIT tier's global table has 32-bit entries
+            o4 = *opts;
+            o4.entry_bytes = 4;
+        }
+        rc = compile_table(patterns, lens, n, split ? &o4 : opts, *t);
+        if (rc == AC_OK && split && !split_table(*t, kDefaultCompactBudget)) {
+            set_error("the automaton has no SPLIT encoding for the default shared-memory budget");
+            rc = AC_ERR_TOO_LARGE;
+        }
         if (rc == AC_OK && opts && opts->tier == AC_TIER_COMPACT && !compact_table(*t, kDefaultCompactBudget)) {
             set_error("the automaton does not fit the COMPACT shared-memory encoding");
             rc = AC_ERR_TOO_LARGE;
@@ -761,6 +840,17 @@ static void fill_info(const ac_table &t, ac_stt_info *info) {
     info->stride = t.stride2 ? 2 : 1;
     info->stride2_cols = t.stride2;
     info->stt2_bytes = (uint64_t)t.stt2.size() * 4;
+    info->split_dense = t.s_dense;
+    info->split_records = t.s_rec;
+    info->split_dstride = t.s_dstride;
+    info->split_cold_records = t.s_cold_rec;
+    info->split_bytes = t.split.size();
+}
+
+ac_status ac_table_export_split(const ac_table *t, void *blob) {
+    if (!t || t->split.empty() || !blob) return AC_ERR_INVALID_ARG;
+    std::memcpy(blob, t->split.data(), t->split.size());
+    return AC_OK;
 }
 
 ac_status ac_table_export_stride2(const ac_table *t, uint32_t *tab) {
@@ -808,7 +898,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
         set_error("the device scan needs the reversed automaton (forward=0)");
         return AC_ERR_INVALID_ARG;
     }
-    if (opts && opts->tier > AC_TIER_COMPACT) {
+    if (opts && opts->tier > AC_TIER_SPLIT) {
         set_error("unknown tier");
         return AC_ERR_INVALID_ARG;
     }
@@ -817,6 +907,12 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     if (rc != AC_OK) return rc;
     ac_stt *h = new (std::nothrow) ac_stt();
     if (!h) return AC_ERR_NO_MEMORY;
+    ac_build_opts o4;
+    if (opts && opts->tier == AC_TIER_SPLIT) {  // the SPLIT tier's global table has 32-bit entries
+        o4 = *opts;
+        o4.entry_bytes = 4;
+        opts = &o4;
+    }
     try {
         rc = compile_table(patterns, lens, n, opts, h->host);
     } catch (...) {
@@ -826,7 +922,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
         delete h;
         return rc;
     }
-    const ac_table &t = h->host;
+    ac_table &t = h->host;
     if ((uint64_t)t.n_states * t.row_stride >= (1ull << 32)) {
         delete h;
         set_error("STT has >= 2^32 entries");
@@ -844,10 +940,36 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     // measured (scripts/sweep.py): an L1-cached global table beats a shared-memory
     // prefix reached through generic loads, so AUTO never picks HYBRID
     const size_t cbudget = stt_budget(h, kLeanVariant);
+    const uint32_t want_stride = opts ? opts->stride : 0;
     if (tier == AC_TIER_AUTO) {
         if (stt_bytes <= budget) tier = AC_TIER_SMEM;
         else if (compact_table(h->host, cbudget)) tier = AC_TIER_COMPACT;
-        else tier = AC_TIER_GLOBAL;
+        // small alphabets (DNA): the L1/L2 table with two bytes per lookup
+        else if (t.n_classes <= 8 && want_stride != 1 && t.entry_bytes == 4) tier = AC_TIER_GLOBAL;
+        else tier = AC_TIER_SPLIT;
+    }
+    if (tier == AC_TIER_SPLIT) {
+        if (t.entry_bytes != 4) {  // the cold states need the 32-bit global table: rebuild it so
+            ac_build_opts o = opts ? *opts : ac_build_opts{sizeof(ac_build_opts), 0, 0, 0, 0, 0};
+            o.entry_bytes = 4;
+            ac_table t4;
+            try {
+                rc = compile_table(patterns, lens, n, &o, t4);
+            } catch (...) {
+                rc = AC_ERR_NO_MEMORY;
+            }
+            if (rc != AC_OK) {
+                delete h;
+                return rc;
+            }
+            h->host = std::move(t4);
+        }
+        if (!split_table(h->host, cbudget)) {
+            delete h;
+            set_error("the automaton has no SPLIT encoding for the shared-memory budget");
+            return AC_ERR_TOO_LARGE;
+        }
+        hot = h->host.s_dense + h->host.s_rec;
     }
     if (tier == AC_TIER_COMPACT) {
         if (h->host.compact.empty() && !compact_table(h->host, cbudget)) {
@@ -864,6 +986,8 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             return AC_ERR_TOO_LARGE;
         }
         hot = t.n_states;
+    } else if (tier == AC_TIER_SPLIT) {
+        // set above
     } else if (tier == AC_TIER_HYBRID) {
         uint32_t cap_rows = (uint32_t)(budget / row_bytes);
         if (hot == 0 || hot > cap_rows) hot = cap_rows;
@@ -875,7 +999,6 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     h->tier = tier;
     h->hot_rows = hot;
     // NEXT-4: two bytes per lookup for small alphabets on the L1/L2 tier
-    const uint32_t want_stride = opts ? opts->stride : 0;
     if (want_stride > 2) {
         delete h;
         set_error("stride must be 0, 1 or 2");
@@ -900,6 +1023,12 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     };
     cudaError_t e = cudaSetDevice(device);
     if (e != cudaSuccess) return fail(e, "cudaSetDevice");
+    if (!t.split.empty() && tier == AC_TIER_SPLIT) {
+        if ((e = cudaMalloc(&h->d_split, (t.split.size() + 15) / 16 * 16)) != cudaSuccess)
+            return fail(e, "cudaMalloc(split)");
+        if ((e = cudaMemcpy(h->d_split, t.split.data(), t.split.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
+            return fail(e, "H2D split");
+    }
     const std::vector<uint8_t> &blob = tier == AC_TIER_COMPACT ? t.compact : t.stt;
     const size_t stt_alloc = (blob.size() + 15) / 16 * 16 + 16;
     if ((e = cudaMalloc(&h->d_stt, stt_alloc)) != cudaSuccess) return fail(e, "cudaMalloc(stt)");
@@ -928,7 +1057,6 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     if ((e = cudaMalloc(&h->d_lens, nl * 4)) != cudaSuccess) return fail(e, "cudaMalloc(lens)");
     if (!t.lens.empty() && (e = cudaMemcpy(h->d_lens, t.lens.data(), t.lens.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
         return fail(e, "H2D lens");
-    keep_pool(device);
     if (prev >= 0 && prev != device) cudaSetDevice(prev);
     *out = h;
     return AC_OK;
@@ -1001,8 +1129,9 @@ ac_status ac_match_shard(const ac_stt *stt, const uint8_t *d_text, uint64_t n_ow
         return AC_ERR_INVALID_ARG;
     }
     cudaStream_t s = static_cast<cudaStream_t>(stream);
+    DeviceGuard guard(stt->device);  // the result word lives on the STT's device
     ac_result *d_res = nullptr;
-    AC_CUDA(cudaMallocAsync(&d_res, sizeof(ac_result), s), "cudaMallocAsync(result)");
+    AC_CUDA(ws_alloc(reinterpret_cast<void **>(&d_res), sizeof(ac_result), s, stt->device), "cudaMallocAsync(result)");
     ac_status rc = ac_match_async(stt, d_text, n_owned, n_halo, base, d_out, cap, d_res, stream, nullptr);
     if (rc == AC_OK) rc = finish_sync(d_res, count, s);
     cudaFreeAsync(d_res, s);

@@ -36,6 +36,12 @@ struct ac_table {
     std::vector<uint8_t> compact;
     std::vector<uint32_t> c_perm;              // compact id -> BFS id
 
+    // SPLIT tier (ac_split.cpp): dense rows for BFS ids [0, s_dense) (s_dstride
+    // u16 entries each), then s_rec 8-byte records for ids [s_dense, s_dense +
+    // s_rec); every other state is read from the global 32-bit table
+    uint32_t s_dense = 0, s_rec = 0, s_dstride = 0, s_cold_rec = 0;
+    std::vector<uint8_t> split;
+
     // two-byte table (NEXT-4), built by stride2_table(): row s, column
     // c1 * n_classes + c2 -> delta(delta(s,c1),c2) | final flag << 31 |
     // middle flag << 30; rows padded to an odd number of words
@@ -51,6 +57,7 @@ struct ac_stt {
     uint32_t hot_rows = 0;
     void *d_stt = nullptr;           // entries
     uint32_t *d_stt2 = nullptr;      // two-byte table (NEXT-4) or NULL
+    void *d_split = nullptr;         // SPLIT tier: the shared-memory part (dense rows + records)
     uint8_t *d_class_map = nullptr;  // 256 B
     uint32_t *d_out_off = nullptr;
     uint32_t *d_out_ids = nullptr;
@@ -65,4 +72,5 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
                         const ac_build_opts *opts, ac_table &t);
 bool compact_table(ac_table &t, size_t budget);
 bool stride2_table(ac_table &t, size_t max_bytes);
+bool split_table(ac_table &t, size_t budget);
 }  // namespace acx

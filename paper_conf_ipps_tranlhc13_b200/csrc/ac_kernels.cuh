@@ -34,7 +34,9 @@
 //
 // STT tiers: SMEM (whole table staged once per CTA),
 // HYBRID (BFS-prefix rows in shared memory, the rest through L1/L2 with a
-// generic load), GLOBAL (L1/L2 only).
+// generic load), GLOBAL (L1/L2 only), COMPACT (dense rows + default-transition
+// records, all in shared memory), SPLIT (COMPACT-like hot part in shared
+// memory, the cold states through L1/L2).
 #pragma once
 
 #include <type_traits>
@@ -67,7 +69,8 @@ __device__ __forceinline__ void stage_tables(uint8_t *s_cmap, E *s_stt, const St
     uint4 *d4 = reinterpret_cast<uint4 *>(s_cmap);
     for (int i = threadIdx.x; i < 16; i += blockDim.x) d4[i] = __ldg(c4 + i);
     const size_t words = ((size_t)st.smem_bytes + 15) / 16;
-    const uint4 *src = reinterpret_cast<const uint4 *>(st.stt);
+    // SPLIT stages its own blob (hot rows + records); the others a prefix of the table
+    const uint4 *src = reinterpret_cast<const uint4 *>(st.sblob ? st.sblob : st.stt);
     uint4 *dst = reinterpret_cast<uint4 *>(s_stt);
     for (size_t i = threadIdx.x; i < words; i += blockDim.x) dst[i] = __ldg(src + i);
 }
@@ -77,8 +80,8 @@ __device__ __forceinline__ uint32_t stt_load(const E *s_stt, const E *g_stt, uin
                                              uint32_t idx) {
     if constexpr (TIER == AC_TIER_SMEM) {
         return s_stt[idx];
-    } else if constexpr (TIER == AC_TIER_GLOBAL) {
-        return __ldg(g_stt + idx);
+    } else if constexpr (TIER == AC_TIER_GLOBAL || TIER == AC_TIER_SPLIT) {
+        return __ldg(g_stt + idx);  // (SPLIT: the output summaries live in the global table)
     } else {
         // HYBRID: two predicated loads, one per address space.  (A generic
         // load would send the shared-memory lanes through the L1TEX tag
@@ -139,6 +142,47 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
     return sp ? (need ? e3 : ex) : lo;
 }
 
+// SPLIT tier (ac_split.cpp): delta(s, cls) as a 32-bit entry (BFS id | flag
+// << 31).  Dense rows (s < s_dense) and 8-byte records (s < s_dense + s_rec)
+// are in shared memory; cold states, cold records (fd = 0xFFFF) and escaped
+// 16-bit entries (0xFFFF: next id >= 32767) read the global table through
+// L1/L2.  Every load is predicated, so lanes in different parts of the
+// automaton never diverge; the cold lanes' global load is issued first, in
+// parallel with the shared-memory loads.
+__device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
+    const uint32_t in_d = s < st.s_dense;
+    const uint32_t in_w = (s - st.s_dense) < st.s_rec;
+    const uint32_t cold = (in_d | in_w) ^ 1u;
+    const uint64_t ga = reinterpret_cast<uint64_t>(static_cast<const uint32_t *>(st.stt)) +
+                        ((uint64_t)s * st.stride + cls) * 4u;
+    uint32_t g = 0;
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u32 %0, [%1];\n\t}"
+                 : "+r"(g)
+                 : "l"(ga), "r"(cold));
+    uint32_t lo = base + s * st.s_row_bytes + cls * 2u;  // dense entry (s, cls)
+    uint32_t hi = base + st.s_rec_x0 + s * 8u;           // record of s
+    asm("{\n\t.reg .pred p, q;\n\tsetp.ne.u32 p, %2, 0;\n\tsetp.ne.u32 q, %3, 0;\n\t"
+        "@p ld.shared.v2.u32 {%0, %1}, [%1];\n\t"
+        "@q ld.shared.u16 %0, [%0];\n\t}"
+        : "+r"(lo), "+r"(hi)
+        : "r"(in_w), "r"(in_d));
+    // record: lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
+    const uint32_t fd = lo & 0xFFFFu;
+    const uint32_t h1 = ((lo >> 16) & 0xFFu) == cls, h2 = (lo >> 24) == cls;
+    const uint32_t ovf = in_w & (fd == 0xFFFFu ? 1u : 0u);
+    const uint32_t need = in_w & ((h1 | h2 | ovf) ^ 1u);
+    uint32_t e3 = base + fd * st.s_row_bytes + cls * 2u;  // dense entry (fd, cls)
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
+        : "+r"(e3)
+        : "r"(need));
+    const uint32_t e16 = in_d ? lo : h1 ? (hi & 0xFFFFu) : h2 ? (hi >> 16) : e3;
+    const uint32_t esc = (cold ^ 1u) & ((e16 == 0xFFFFu ? 1u : 0u) | ovf);
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u32 %0, [%1];\n\t}"
+                 : "+r"(g)
+                 : "l"(ga), "r"(esc));
+    return (cold | esc) ? g : ((e16 >> 1) | (e16 << 31));
+}
+
 // Entry -> next state and output flag.
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t state_of(uint32_t e, const SttView &st) {
@@ -159,6 +203,8 @@ template <typename E, int TIER>
 __device__ __forceinline__ uint32_t next_entry(const E *s_stt, const SttView &st, uint32_t s, uint32_t cls) {
     if constexpr (TIER == AC_TIER_COMPACT) {
         return compact_next(smem_u32(s_stt), st, s, cls);
+    } else if constexpr (TIER == AC_TIER_SPLIT) {
+        return split_next(smem_u32(s_stt), st, s, cls);
     } else {
         return stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
     }
@@ -203,7 +249,7 @@ __device__ __forceinline__ uint32_t out_payload(const E *s_stt, const SttView &s
         const uint32_t *gp = reinterpret_cast<const uint32_t *>(static_cast<const E *>(st.stt) + idx);
         if constexpr (TIER == AC_TIER_SMEM) {
             return *sp;
-        } else if constexpr (TIER == AC_TIER_GLOBAL) {
+        } else if constexpr (TIER == AC_TIER_GLOBAL || TIER == AC_TIER_SPLIT) {
             return __ldg(gp);
         } else {
             return *((s < st.smem_rows) ? sp : gp);
@@ -254,7 +300,7 @@ __device__ __forceinline__ uint2 out_info_pred(const E *s_stt, const SttView &st
             const E *g = static_cast<const E *>(st.stt);
             const E *base = (TIER == AC_TIER_HYBRID && s < st.smem_rows) ? s_stt : g;
             const uint64_t pc = reinterpret_cast<uint64_t>(base + ic), pp = reinterpret_cast<uint64_t>(base + ip);
-            if constexpr (TIER == AC_TIER_GLOBAL) {
+            if constexpr (TIER == AC_TIER_GLOBAL || TIER == AC_TIER_SPLIT) {
                 if constexpr (sizeof(E) == 2)
                     asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u16 %0, [%1];\n\t}"
                         : "+r"(c)
@@ -624,9 +670,9 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
 // Epilogue of the single emitting pass when the main region starts the list
 // (no head chains): a CTA's chains are consecutive in canonical order, so
 // the CTA needs only the match total of the CTAs before it -- a decoupled
-// look-back over one word per CTA (CTAs are dispatched in index order, so
-// every predecessor is running or done; warp 0 reads 32 predecessors per
-// step) -- to write every chain's end offset.  This replaces the k_offsets
+// look-back over one word per CTA (tile indices come from an atomic ticket
+// taken at CTA start, so every predecessor is running or done; warp 0 reads
+// 32 predecessors per step) -- to write every chain's end offset.  This replaces the k_offsets
 // launch.  Shared memory for the exchange is the warps' own (finished) TMA
 // ring slots.
 __device__ __forceinline__ uint64_t ld_acquire_u64(const unsigned long long *p) {
@@ -640,8 +686,8 @@ __device__ __forceinline__ void st_release_u64(unsigned long long *p, uint64_t v
 
 template <int K>
 __device__ __forceinline__ void place_chains(const ScanOut &so, const StagedGeom &g, uint8_t *wring, uint8_t *ring,
-                                             int warp_ring, int warps, uint64_t row0, const uint32_t (&cnt)[K],
-                                             const bool (&live)[K]) {
+                                             int warp_ring, int warps, uint32_t tile, uint64_t row0,
+                                             const uint32_t (&cnt)[K], const bool (&live)[K]) {
     const int lane = threadIdx.x & 31;
     // warp-level inclusive scan in canonical chain order (k major, lane minor)
     uint64_t incl[K];
@@ -665,11 +711,11 @@ __device__ __forceinline__ void place_chains(const ScanOut &so, const StagedGeom
         uint64_t tot = 0;
         for (int w = 0; w < warps; w++) tot += reinterpret_cast<uint64_t *>(ring + w * warp_ring)[0];
         uint64_t prefix = 0;
-        if (blockIdx.x == 0) {
+        if (tile == 0) {
             if (lane == 0) st_release_u64(&so.tile_state[0], LB_INC | tot);
         } else {
-            if (lane == 0) st_release_u64(&so.tile_state[blockIdx.x], LB_AGG | tot);
-            int64_t p = (int64_t)blockIdx.x - 1;  // nearest predecessor of the window
+            if (lane == 0) st_release_u64(&so.tile_state[tile], LB_AGG | tot);
+            int64_t p = (int64_t)tile - 1;  // nearest predecessor of the window
             while (true) {
                 const int64_t idx = p - lane;
                 uint64_t st = idx >= 0 ? ld_acquire_u64(&so.tile_state[idx]) : LB_INC;  // before CTA 0: 0
@@ -683,7 +729,7 @@ __device__ __forceinline__ void place_chains(const ScanOut &so, const StagedGeom
                 if (inc) break;
                 p -= 32;
             }
-            if (lane == 0) st_release_u64(&so.tile_state[blockIdx.x], LB_INC | (prefix + tot));
+            if (lane == 0) st_release_u64(&so.tile_state[tile], LB_INC | (prefix + tot));
         }
         if (lane == 0)  // exclusive prefix of every warp, into its slot (word 1)
             for (int w = 0; w < warps; w++) {
@@ -706,7 +752,10 @@ struct StagedShape {
     static constexpr int SLOT = ROWS * W;             // bytes per ring slot
     static constexpr int WARP_RING = NST * SLOT;
     static constexpr int RING = WARPS * WARP_RING;
-    static constexpr int BARS = (WARPS * NST * 8 + 15) / 16 * 16;
+    // mbarriers, then one 16-byte word for the CTA's tile ticket (dynamic
+    // shared memory: a static __shared__ variable would push the 1024-B
+    // aligned dynamic base by a whole 1 KB)
+    static constexpr int BARS = (WARPS * NST * 8 + 16 + 15) / 16 * 16;
     static constexpr uint32_t SWZ = !SWIZZLE ? 0u : W == 128 ? 7u : W == 64 ? 3u : W == 32 ? 1u : 0u;
     static_assert(ROWS <= 256, "TMA box rows");
     static_assert(W == 16 || W == 32 || W == 64 || W == 128, "tile width");
@@ -728,19 +777,23 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     E *s_stt = reinterpret_cast<E *>(s_cmap + 256);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
+    // in-kernel placement (look-back) takes the CTA's tile from a ticket
+    const bool place = MODE == MODE_EMIT_OPT && so.tile_state != nullptr;
+    uint32_t &s_tile = *reinterpret_cast<uint32_t *>(bars + WARPS * NST);
     if (threadIdx.x < WARPS * NST) mbar_init(&bars[threadIdx.x], 1);
     if (threadIdx.x == 0) {
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
+        s_tile = place ? atomicAdd(so.ticket, 1u) : blockIdx.x;
     }
     stage_tables<E>(s_cmap, s_stt, st);
-    __syncthreads();  // the only CTA-wide barrier: tables staged, barriers initialised
+    __syncthreads();  // the only CTA-wide barrier: tables staged, barriers initialised, tile taken
     if constexpr (MODE == MODE_EMIT) {
         if (so.res->status != AC_OK) return;  // capacity exceeded: write nothing
     }
-    const uint64_t row0 = (uint64_t)blockIdx.x * (WARPS * Sh::ROWS) + (uint64_t)warp * Sh::ROWS;
+    const uint32_t tile = s_tile;
+    const uint64_t row0 = (uint64_t)tile * (WARPS * Sh::ROWS) + (uint64_t)warp * Sh::ROWS;
     // in-kernel placement ends with CTA barriers: idle warps stay (no tiles)
-    const bool place = MODE == MODE_EMIT_OPT && so.tile_state != nullptr;
     const bool idle = row0 >= g.n_chains;
     if (idle && !place) return;  // idle warp (no later CTA barrier)
 
@@ -979,7 +1032,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
             if (live[k]) so.chain_counts[g.chain0 + row0 + k * 32 + lane] = cnt[k];
     }
     if constexpr (MODE == MODE_EMIT_OPT) {
-        if (place) place_chains<K>(so, g, wring, ring, Sh::WARP_RING, WARPS, row0, cnt, live);
+        if (place) place_chains<K>(so, g, wring, ring, Sh::WARP_RING, WARPS, tile, row0, cnt, live);
     }
 
     if constexpr (MODE == MODE_COUNT_TOTAL) {
@@ -1142,6 +1195,13 @@ template <int TIER>
 cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtensorMap &tmap, const uint8_t *mtext,
                                const SttView &st, const StagedGeom &g, const ScanOut &so, size_t smem_stt,
                                cudaStream_t stream) {
+    if constexpr (TIER == AC_TIER_SPLIT) {  // the cold part is the 32-bit global table
+        if (eb != 4) return cudaErrorInvalidValue;
+        return with_mode(mode, [&](auto m) {
+            return launch_staged_m<uint32_t, TIER, decltype(m)::value>(variant, tmap, mtext, st, g, so, smem_stt,
+                                                                       stream);
+        });
+    }
     if (eb == 2)
         return with_mode(mode, [&](auto m) {
             return launch_staged_m<uint16_t, TIER, decltype(m)::value>(variant, tmap, mtext, st, g, so, smem_stt,

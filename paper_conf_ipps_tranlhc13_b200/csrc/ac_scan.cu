@@ -19,7 +19,7 @@ const StagedConfig &staged_variant(int v) { return kVariants[v - 1]; }
 
 size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt) {
     const size_t ring = (size_t)cfg.warps * cfg.stages * 32 * cfg.k * cfg.width;
-    const size_t bars = ((size_t)cfg.warps * cfg.stages * 8 + 15) / 16 * 16;
+    const size_t bars = ((size_t)cfg.warps * cfg.stages * 8 + 16 + 15) / 16 * 16;  // + the tile ticket word
     // swizzled tiles (W >= 32) align the ring to the 1024-B swizzle atom at run time
     const size_t align = cfg.swizzle && cfg.width >= 32 ? 1024 : 0;
     return align + ring + bars + 256 + smem_stt;
@@ -43,6 +43,7 @@ cudaError_t launch_scan_staged(int mode, uint32_t eb, uint32_t tier, int variant
         case AC_TIER_SMEM: return launch_staged_tier<AC_TIER_SMEM>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
         case AC_TIER_HYBRID: return launch_staged_tier<AC_TIER_HYBRID>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
         case AC_TIER_COMPACT: return launch_staged_tier<AC_TIER_COMPACT>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
+        case AC_TIER_SPLIT: return launch_staged_tier<AC_TIER_SPLIT>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
         default: return launch_staged_tier<AC_TIER_GLOBAL>(mode, eb, variant, tmap, mtext, st, g, so, smem_stt, stream);
     }
 }

@@ -40,6 +40,12 @@ struct SttView {
     // two-byte table (NEXT-4): row s, column c1 * n_classes + c2; NULL = off
     const uint32_t *stt2;
     uint32_t stride2, n_classes;
+    // SPLIT tier (ac_split.cpp): shared-memory part staged from `sblob` --
+    // dense rows of BFS ids [0, s_dense) at s * s_row_bytes, 8-byte records
+    // of ids [s_dense, s_dense + s_rec) at s_rec_x0 + 8 s (biased, wraps);
+    // `stt` stays the full 32-bit table for the cold states
+    const void *sblob;
+    uint32_t s_dense, s_rec, s_row_bytes, s_rec_x0;
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.
@@ -66,10 +72,15 @@ struct ScanOut {
     uint32_t nbits;
     // MODE_EMIT_OPT, staged kernel, when the main region starts the list
     // (NULL = off): each CTA publishes its match total in tile_state
-    // [blockIdx.x] (decoupled look-back) and writes the end offset of each of
+    // [its ticket] (decoupled look-back) and writes the end offset of each of
     // its chains into chain_end_w -- the offset scan runs inside the scan
     unsigned long long *tile_state;
     uint64_t *chain_end_w;
+    // with tile_state: zeroed counter from which each staged CTA takes its
+    // tile index (an atomic ticket), so every look-back predecessor of a
+    // running CTA is itself running or done -- CUDA does not promise that
+    // CTAs start in blockIdx order
+    unsigned int *ticket;
 };
 
 // Decoupled look-back words: 2-bit flag (aggregate / inclusive prefix) + value.

@@ -56,8 +56,18 @@ def plan_shards(n: int, world: int, maxlen: int, align: int = 16) -> list[Shard]
     return [Shard(g, bounds[g], bounds[g + 1], min(H, n - bounds[g + 1])) for g in range(world)]
 
 
-def allreduce_count(count: int, device, group=None) -> int:
-    t = torch.tensor([count], dtype=torch.int64, device=device)
+def _comm_device(t: torch.Tensor, group=None):
+    """gloo moves host tensors (CPU tests, or GPU ranks without NCCL); NCCL
+    moves device tensors over NVLink/NVSwitch."""
+    return torch.device("cpu") if dist.get_backend(group) == "gloo" else t.device
+
+
+def allreduce_count(count, device, group=None) -> int:
+    """Global match count: all_reduce(SUM) of the per-rank counts (an int or a
+    1-element int64 tensor)."""
+    t = count.reshape(1).to(torch.int64) if isinstance(count, torch.Tensor) else \
+        torch.tensor([count], dtype=torch.int64, device=device)
+    t = t.to(_comm_device(t, group)).clone()
     dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
     return int(t.item())
 
@@ -65,32 +75,53 @@ def allreduce_count(count: int, device, group=None) -> int:
 def allgatherv(records: torch.Tensor, group=None) -> torch.Tensor:
     """Concatenate every rank's 1-D int64 tensor in rank order (on all ranks)."""
     world = dist.get_world_size(group)
-    dev = records.device
+    home = records.device
+    dev = _comm_device(records, group)
+    records = records.to(dev)
     n = torch.tensor([records.numel()], dtype=torch.int64, device=dev)
     counts = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in range(world)]
     dist.all_gather(counts, n, group=group)
     counts = [int(c.item()) for c in counts]
     m = max(counts) if counts else 0
     if m == 0:
-        return records.new_empty(0)
+        return records.new_empty(0).to(home)
     padded = torch.full((m,), -1, dtype=torch.int64, device=dev)
     padded[:records.numel()] = records
     out = torch.empty(world * m, dtype=torch.int64, device=dev)
     dist.all_gather_into_tensor(out, padded, group=group)
-    return torch.cat([out[g * m:g * m + c] for g, c in enumerate(counts)])
+    return torch.cat([out[g * m:g * m + c] for g, c in enumerate(counts)]).to(home)
 
 
-def match_sharded(stt, shard_text: torch.Tensor, shard: Shard, *, gather: bool = True, group=None,
-                  stream=None, **knobs):
+def default_capacity(owned: int) -> int:
+    """Count-free output capacity: one record per 8 owned bytes (an output
+    buffer the size of the text).  Enough for the BASELINE configs (<= 0.07
+    matches per byte); a denser shard reports its exact need and is re-run."""
+    return owned // 8 + 64
+
+
+def match_sharded(stt, shard_text: torch.Tensor, shard: Shard, *, out: torch.Tensor | None = None,
+                  gather: bool = True, group=None, stream=None, **knobs):
     """Scan this rank's shard (device tensor holding text[shard.lo : shard.read_hi])
-    and combine.  Returns (global_count, records): the global canonical list
-    when gather=True, else this rank's slice of it (rank-order concatenation
-    of the slices is the global list)."""
-    from . import match  # the CUDA path; no fallback
+    in ONE emitting pass and combine.  Returns (global_count, records): the
+    global canonical list when gather=True, else this rank's slice of it
+    (rank-order concatenation of the slices is the global list).  ``out``:
+    optional int64 device buffer (default: default_capacity)."""
+    from . import AC_ERR_CAPACITY, _check, match_async  # the CUDA path; no fallback
     if shard_text.numel() != shard.read_hi - shard.lo:
         raise ValueError("shard_text must hold text[lo:hi + halo]")
-    c, recs = match(stt, shard_text, n_halo=shard.halo, base=shard.lo, stream=stream, **knobs)
-    total = allreduce_count(c, shard_text.device, group)
+    dev = shard_text.device
+    if out is None:
+        out = torch.empty(default_capacity(shard.owned), dtype=torch.int64, device=dev)
+    res = torch.zeros(2, dtype=torch.int64, device=dev)
+    match_async(stt, shard_text, out, res, n_halo=shard.halo, base=shard.lo, stream=stream, **knobs)
+    c, st = (int(x) for x in res.tolist())
+    if st == AC_ERR_CAPACITY:  # denser than the default bound: exact size, scan again
+        out = torch.empty(max(1, c), dtype=torch.int64, device=dev)
+        match_async(stt, shard_text, out, res, n_halo=shard.halo, base=shard.lo, stream=stream, **knobs)
+        c, st = (int(x) for x in res.tolist())
+    _check(st)
+    recs = out[:c]
+    total = allreduce_count(res[:1], dev, group)
     if gather:
         recs = allgatherv(recs.contiguous(), group)
     return total, recs

@@ -15,6 +15,8 @@ every consumer sees identical bytes.  Seeds are 1000*cfg + 0 (text),
 """
 from __future__ import annotations
 
+import os
+from concurrent.futures import ThreadPoolExecutor
 from dataclasses import dataclass, field
 
 import numpy as np
@@ -40,9 +42,18 @@ def _blocks(n: int, seed: int, fill, block0: int = 0) -> np.ndarray:
     """Allocate n bytes and fill them block by block with fill(rng, view, j);
     the text starts at block ``block0`` of the (endless) seeded stream."""
     out = np.empty(n, dtype=np.uint8)
-    for j, lo in enumerate(range(0, n, BLOCK)):
-        hi = min(n, lo + BLOCK)
-        fill(rng_for(seed, block0 + j), out[lo:hi], block0 + j)
+
+    def one(j):
+        lo = j * BLOCK
+        fill(rng_for(seed, block0 + j), out[lo:min(n, lo + BLOCK)], block0 + j)
+
+    nb = (n + BLOCK - 1) // BLOCK
+    if nb >= 8:  # blocks are independent: fill them on every host core
+        with ThreadPoolExecutor(min(nb, os.cpu_count() or 1)) as ex:
+            list(ex.map(one, range(nb)))
+    else:
+        for j in range(nb):
+            one(j)
     return out
 
 

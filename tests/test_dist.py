@@ -56,8 +56,13 @@ def _worker(rank, world, port, q):
         full = allgatherv(local)
         want = _keys(o, w.text, 0, w.text.size)
         ok = total == want.numel() and torch.equal(full, want)
-        empty = allgatherv(torch.empty(0, dtype=torch.int64) if rank else local)
-        ok = ok and torch.equal(empty, local if rank == 0 else empty)
+        # only rank 0 contributes: every rank must receive exactly rank 0's
+        # slice (each rank recomputes it from the oracle to compare)
+        r0 = _keys(o, w.text[:shards[0].read_hi], 0, shards[0].owned)
+        got0 = allgatherv(torch.empty(0, dtype=torch.int64) if rank else local)
+        ok = ok and torch.equal(got0, r0)
+        # and nobody contributes
+        ok = ok and allgatherv(torch.empty(0, dtype=torch.int64)).numel() == 0
         q.put((rank, bool(ok), total, want.numel()))
     finally:
         dist.destroy_process_group()

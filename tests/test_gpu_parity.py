@@ -174,9 +174,51 @@ def test_c3_hybrid_and_global_tiers():
     w = synth.make("c3", n=(1 << 20) + 5)
     o = Oracle(w.patterns)
     want = oracle_keys(o, w.text)
-    for tier in (ac.TIER_AUTO, ac.TIER_HYBRID, ac.TIER_GLOBAL):
+    assert ac.build(w.patterns).tier_name == "split"  # AUTO for a 131K-state byte dictionary
+    for tier in (ac.TIER_AUTO, ac.TIER_HYBRID, ac.TIER_GLOBAL, ac.TIER_SPLIT):
         stt = ac.build(w.patterns, tier=tier)
         assert_same(gpu_keys(stt, w.text), want)
+        assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED), want)
+
+
+# SPLIT tier: hot rows + records in shared memory, cold states via L1/L2
+@pytest.mark.parametrize("name,n,P", [("c3", (3 << 20) + 11, None), ("c5-english-5000-22", None, None),
+                                      ("c5-english-20000-22", None, None), ("c1", (1 << 20) + 3, None),
+                                      ("c5-snort-1000-21", None, None)])
+def test_split_tier(name, n, P):
+    w = synth.make(name, n=n, n_patterns=P)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns, tier=ac.TIER_SPLIT)
+    assert stt.tier_name == "split" and stt.info["entry_bytes"] == 4 and stt.info["split_bytes"] > 0
+    want = oracle_keys(o, w.text)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED), want)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, chain_bytes=112), want)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_GLOBAL), want)
+
+
+def test_split_tier_escapes_and_cold_records():
+    # a 20K-pattern English dictionary (265K states): records of deep states
+    # point past id 32766 (escaped 16-bit entries) and some need > 2
+    # exceptions (cold records) -- both must fall back to the global table
+    w = synth.make("c5-english-20000-22")
+    stt = ac.build(w.patterns, tier=ac.TIER_SPLIT)
+    T = ac.compile_table(w.patterns, split=True)
+    assert T.info["split_cold_records"] > 0
+    D, W, ds = T.info["split_dense"], T.info["split_records"], T.info["split_dstride"]
+    rec = T.split[D * ds * 2:D * ds * 2 + W * 8].view(np.uint32).reshape(-1, 2)
+    assert ((rec[:, 1] & 0xFFFF) == 0xFFFF).any() or ((rec[:, 1] >> 16) == 0xFFFF).any()
+    o = Oracle(w.patterns)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED), oracle_keys(o, w.text))
+
+
+@pytest.mark.parametrize("variant", [1, 3, 4, 7, 9])
+def test_split_tier_variants(variant):
+    # a smaller byte dictionary so the split part also fits the fat-ring variants
+    w = synth.make("c3", n=(2 << 20) + 4321, n_patterns=1500)
+    o = Oracle(w.patterns)
+    stt = ac.build(w.patterns, tier=ac.TIER_SPLIT)
+    want = oracle_keys(o, w.text)
+    assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
 
 
 @pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7, 8])
@@ -440,33 +482,90 @@ def test_determinism():
 
 
 # ------------------------------------------------- full BASELINE.json sizes
-def _windows(n, k, width, seed):
-    rng = np.random.default_rng(seed)
-    los = [0, n - width] + rng.integers(0, n - width, size=k - 2).tolist()
-    return [(int(lo), int(lo) + width) for lo in los]
+# Every config at its full size, compared with the oracle over the WHOLE text
+# (the oracle runs as start-owned windows on every host core, P:163-164 one
+# level up): the complete canonical list where the oracle can hold it (C2,
+# C3), else the full count plus the order-free multiset digest (count, sum,
+# xor of splitmix64(start << 24 | pid)) computed independently on each side
+# (SURVEY 8(c) "GPU parity").  The list comes from the launch configuration
+# bench.py times (auto tier, auto kernel, single emitting pass).
+_M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
 
 
-def _check_windows(o, text_np, recs_np, windows):
-    s = recs_np >> 24
-    for lo, hi in windows:
-        a, b = np.searchsorted(s, lo, "left"), np.searchsorted(s, hi, "left")
-        assert_same(recs_np[a:b], oracle_keys(o, text_np, lo, hi))
+def _np_mix64(x: np.ndarray) -> np.ndarray:
+    """splitmix64 over a uint64 array (wrapping arithmetic), test-side copy."""
+    with np.errstate(over="ignore"):
+        z = x + np.uint64(0x9E3779B97F4A7C15)
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        return z ^ (z >> np.uint64(31))
 
 
-@pytest.mark.slow
-@pytest.mark.parametrize("name,width,k", [("c2", 1 << 18, 8), ("c3", 1 << 17, 5), ("c4", 1 << 18, 6)])
-def test_full_size_sampled(name, width, k):
+def digest_keys(keys: np.ndarray):
+    """(count, sum mod 2^64, xor) of splitmix64 over the records (uint64 view)."""
+    k = keys.view(np.uint64)
+    c, sm, x = int(k.size), 0, 0
+    for lo in range(0, k.size, 1 << 26):
+        h = _np_mix64(k[lo:lo + (1 << 26)])
+        with np.errstate(over="ignore"):
+            sm = (sm + int(h.sum(dtype=np.uint64))) & ((1 << 64) - 1)
+        x ^= int(np.bitwise_xor.reduce(h)) if h.size else 0
+    return c, sm, x
+
+
+def test_np_mix64_known_values():
+    assert int(_np_mix64(np.array([0], np.uint64))[0]) == 0xE220A8397B1DCDAF
+
+
+def _full_list(name):
     w = synth.make(name)
-    o = Oracle(w.patterns)
     stt = ac.build(w.patterns)
     t = torch.from_numpy(w.text).cuda()
     c, recs = ac.match(stt, t)
-    r = recs.cpu().numpy()
-    assert c == r.size and (c == 0 or np.all(r[1:] > r[:-1]))  # canonical and duplicate free
-    # count-only agrees with the list; the staged and global-only kernels agree
     assert ac.count(stt, t) == c
-    _check_windows(o, w.text, r, _windows(w.text.size, k, width, 7))
+    r = recs.cpu().numpy()
     del t, recs
+    torch.cuda.empty_cache()
+    return w, stt, c, r
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["c2", "c3"])
+def test_full_size_whole_list(name):
+    w, stt, c, r = _full_list(name)
+    o = Oracle(w.patterns)
+    ends, pids = o.match_parallel(w.text)
+    starts = ends.astype(np.int64) - o.lens[pids].astype(np.int64) + 1
+    assert_same(r, (starts << 24) | pids.astype(np.int64))
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["c4", "c5-english-5000-30", "c5-snort-10000-30"])
+def test_full_size_count_and_digest(name):
+    w, stt, c, r = _full_list(name)
+    assert c == r.size and (c == 0 or np.all(r[1:] > r[:-1]))  # canonical, duplicate free
+    o = Oracle(w.patterns)
+    assert digest_keys(r) == o.digest_parallel(w.text)
+
+
+@pytest.mark.slow
+def test_full_size_adversarial_runs_4gib():
+    # C5 adversarial a^n with {a^1..a^32} at n = 2^32: count = K n - K(K-1)/2
+    # (closed form P4-i); the 1.1 TB list cannot be held, so count mode over
+    # the whole text plus the list of sampled sub-texts via the shard API
+    K, n = 32, 1 << 32
+    stt = ac.build([b"a" * k for k in range(1, K + 1)])
+    t = torch.full((n,), ord("a"), dtype=torch.uint8, device="cuda")
+    assert ac.count(stt, t) == K * n - K * (K - 1) // 2
+    for lo in (0, (1 << 31) + 7, n - 4096):
+        hi = min(n, lo + 4096)
+        halo = min(K - 1, n - hi)
+        c, recs = ac.match(stt, t[lo:hi + halo], n_halo=halo, base=lo)
+        r = recs.cpu().numpy()
+        per = np.minimum(K, n - np.arange(lo, hi))
+        assert c == int(per.sum())
+        assert np.array_equal(r >> 24, np.repeat(np.arange(lo, hi), per))
+    del t
 
 
 @pytest.mark.slow

@@ -199,7 +199,7 @@ def test_compact_encoding_equals_dense(which):
         assert count == len(outs) and payload == (outs[0] if count == 1 else int(t.out_off[s]))
     # fits next to the lean staged variant's ring (32 warps x 2 slots x 512 B, unswizzled:
     # no alignment pad), its mbarriers, the class map and 128 B of slack
-    assert d["compact_bytes"] <= 232448 - (32 * 2 * 512 + 512 + 256) - 128
+    assert d["compact_bytes"] <= 232448 - (32 * 2 * 512 + 512 + 16 + 256) - 128
     if which == "c2":
         assert S > 15000 and d["stt_bytes"] > 1_000_000  # the dense table would not fit
 
@@ -271,3 +271,59 @@ def test_compact_rejects_wide_alphabets():
     wide = [bytes([b, (b * 7) % 256]) for b in range(200)]
     with pytest.raises(ac.AcError):
         ac.compile_table(wide, compact=True)
+
+
+def _decode_split(t):
+    """The SPLIT lookup rule of include/ac.h, vectorised over the states in
+    shared memory: E[s, c] = 32-bit entry (BFS id | flag << 31) where the
+    shared-memory part answers, -1 where the global table must (cold record or
+    escaped entry)."""
+    d = t.info
+    C = d["n_classes"]
+    D, W, ds = d["split_dense"], d["split_records"], d["split_dstride"]
+    blob = t.split
+    dense = blob[:D * ds * 2].view(np.uint16).reshape(D, ds)[:, :C].astype(np.int64)
+    rec = blob[D * ds * 2:D * ds * 2 + W * 8].view(np.uint32).reshape(-1, 2).astype(np.int64)
+    fd = rec[:, 0] & 0xFFFF
+    c1, c2 = (rec[:, 0] >> 16) & 0xFF, rec[:, 0] >> 24
+    t1, t2 = rec[:, 1] & 0xFFFF, rec[:, 1] >> 16
+    cls = np.arange(C)[None, :]
+    cold = fd == 0xFFFF
+    fb = dense[np.where(cold, 0, fd)]
+    sparse = np.where(cls == c1[:, None], t1[:, None], np.where(cls == c2[:, None], t2[:, None], fb))
+    sparse[cold] = 0xFFFF
+    e16 = np.concatenate([dense, sparse])
+    E = (e16 >> 1) | ((e16 & 1) << 31)
+    return np.where(e16 == 0xFFFF, -1, E), int(cold.sum())
+
+
+@pytest.mark.parametrize("which", ["c3", "english5k", "tiny"])
+def test_split_encoding_equals_dense(which):
+    """Every transition the SPLIT shared-memory part answers equals the dense
+    table's delta; the rest are marked for the global table."""
+    import synth
+    if which == "tiny":
+        pats = [b"he", b"she", b"his", b"hers", b"h", b"hershey"]
+    elif which == "c3":
+        pats = synth.patterns_snort(10000, 3001)
+    else:
+        pats = synth.make("c5-english-5000-22").patterns
+    t = ac.compile_table(pats, split=True)
+    d = t.info
+    assert d["entry_bytes"] == 4 and d["split_bytes"] > 0
+    C, D, W = d["n_classes"], d["split_dense"], d["split_records"]
+    E, n_cold = _decode_split(t)
+    assert n_cold == d["split_cold_records"]
+    want = t.stt[:D + W, :C].astype(np.int64)
+    ok = E >= 0
+    assert np.array_equal(E[ok], want[ok])
+    # escapes only where the next id does not fit 15 bits, or cold records
+    esc_dense = ~ok[:D]
+    assert ((want[:D][esc_dense] & 0x7FFFFFFF) >= 32767).all()
+    assert D >= 1
+    # fits next to the lean staged variant's ring
+    assert d["split_bytes"] <= 232448 - (32 * 2 * 512 + 512 + 16 + 256) - 128
+    if which == "c3":
+        # depth <= 1 dense (root + one state per used last byte), depth-2 states as records
+        assert D == 1 + len({p[-1] for p in pats})
+        assert W >= 7000 and d["split_cold_records"] < W // 10
