@@ -147,13 +147,24 @@ typedef struct {
     uint32_t stride;       /* 1 or 2 (two-byte table present)                */
     uint32_t stride2_cols; /* row stride of the two-byte table (C*C, odd)   */
     uint64_t stt2_bytes;
-    /* SPLIT tier (valid when split_bytes != 0): BFS ids [0, split_dense) are
-     * dense rows of split_dstride u16 entries, ids [split_dense, split_dense +
-     * split_records) are 8-byte records {lo32 = fd | c1 << 16 | c2 << 24,
-     * hi32 = t1 | t2 << 16}; a u16 entry is 2 x + flag, or 0xFFFF = read the
-     * global table; split_cold_records of the records are cold (fd 0xFFFF). */
+    /* SPLIT tier (valid when split_bytes != 0): split_dense + 1 dense rows of
+     * split_dstride u16 entries (row r = BFS state r for r < split_dense, the
+     * last one all 0xFFFF), then one 8-byte record per sparse hot state
+     * split_dense <= s < split_records: {lo32 = fd | c1 << 16 | c2 << 24,
+     * hi32 = t1 | t2 << 16}, delta(s, c) = t1 if c == c1, t2 if c == c2, else
+     * row[fd][c]; dense states read row[s][c]; a u16 entry is 2 x + flag, or
+     * 0xFFFF = read the global table; split_cold_records sparse states point
+     * at the 0xFFFF row; states >= split_records are read from the global
+     * table. */
     uint32_t split_dense, split_records, split_dstride, split_cold_records;
     uint64_t split_bytes;
+    /* SPLIT cold records (global memory, split_crec_bytes = 16 x n_states):
+     * w0 = fd | c1 << 16 | c2 << 24, w1 = t1, w2 = t2 (32-bit entries),
+     * w3 = c3 | t3 << 8 (23-bit id, flag in bit 31); fd = 0xFFFF (the
+     * split_cold_full states needing more exceptions, and the dense states)
+     * = read the 32-bit dense table. */
+    uint32_t split_cold_full, reserved2;
+    uint64_t split_crec_bytes;
 } ac_stt_info;
 
 /* Scan variants (SURVEY 8(f) NEXT-1 ablations are selectable here). */
@@ -179,8 +190,8 @@ typedef struct {
                               (0 = auto from cap); chains with more are
                               re-scanned straight into place                 */
     uint32_t two_pass;     /* list mode: 0 = auto: single emitting pass, or
-                              the two passes when cap / chains > ~1K records
-                              (several matches per byte); single pass: chain
+                              the two passes when cap > n (room for more
+                              than one record per text byte); single pass: chain
                               offsets computed inside the staged scan when
                               the text pointer is 16-byte aligned, else by
                               a separate offset scan); 1 = count pass + emit
@@ -195,6 +206,13 @@ typedef struct {
                               and events[2i+1] are recorded on the stream
                               right before / after kernel launch i, so a
                               caller can time each kernel (bench.py)         */
+    uint32_t text_policy;  /* L2 policy of the staged kernel's text loads:
+                              0 = auto (evict-first where the table lives in
+                              L2: GLOBAL, HYBRID, SPLIT), 1 = evict-normal,
+                              2 = evict-first (ablation knob)               */
+    uint32_t stt_policy;   /* SPLIT tier: L2 policy of the cold global-table
+                              loads: 0 = auto, 1 = evict-normal, 2 =
+                              evict-last (keeps cold rows ahead of the text) */
 } ac_match_opts;
 
 /* Per-call device result written by the async entry points. */
@@ -307,8 +325,9 @@ ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm)
  * output(final) != {} | bit 30 = output(middle) != {}. */
 ac_status ac_table_export_stride2(const ac_table *t, uint32_t *tab);
 /* opts->tier == AC_TIER_SPLIT (ac_compile) builds the SPLIT shared-memory
- * part for the default budget (32-bit table); copies its split_bytes. */
-ac_status ac_table_export_split(const ac_table *t, void *blob);
+ * part for the default budget (32-bit table); copies its split_bytes and,
+ * if crec != NULL, the split_crec_bytes of cold records. */
+ac_status ac_table_export_split(const ac_table *t, void *blob, uint32_t *crec);
 void ac_table_free(ac_table *t);
 
 /* ------------------------------------------------------------ diagnostics */

@@ -304,6 +304,30 @@ uint64_t oracle_match_chunked(const ac_oracle *m, const uint8_t *text, uint64_t 
     return count;
 }
 
+/*
+ * Transition counts of the walk of P:55-58 over text[0, n) (SURVEY 8(c)
+ * pin P6, "O(n)"): out[0] = goto transitions (one per input symbol,
+ * the root's self-loop g(0,a) = 0 included), out[1] = failure transitions
+ * (state <- f(state)).  AC'75 bounds the failure transitions by the goto
+ * transitions (each failure move strictly decreases the depth, which each
+ * goto move raises by at most one), so the whole walk is O(n).
+ */
+void oracle_transitions(const ac_oracle *m, const uint8_t *text, uint64_t n, uint64_t *out) {
+    uint64_t gotos = 0, fails = 0;
+    uint32_t state = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        uint8_t a = text[i];
+        while (oracle_goto(m, state, a) == FAIL) {
+            state = m->nodes[state].fail;
+            fails++;
+        }
+        state = (uint32_t)oracle_goto(m, state, a);
+        gotos++;
+    }
+    out[0] = gotos;
+    out[1] = fails;
+}
+
 /* Canonical order (reading R3): start ascending, then pattern id ascending.
  * Each element carries its own start, so the comparator needs no shared state
  * and concurrent calls from several threads are safe. */

@@ -73,6 +73,8 @@ def _load():
         lib.oracle_digest_window.restype = None
         lib.oracle_digest_window.argtypes = [ctypes.c_void_p, _u8p, ctypes.c_uint64, ctypes.c_uint64,
                                              ctypes.c_uint64, ctypes.c_uint64, _u64p]
+        lib.oracle_transitions.restype = None
+        lib.oracle_transitions.argtypes = [ctypes.c_void_p, _u8p, ctypes.c_uint64, _u64p]
         lib.oracle_canonical_sort.restype = ctypes.c_int
         lib.oracle_canonical_sort.argtypes = [ctypes.c_void_p, _u64p, _u32p, ctypes.c_uint64]
         _lib = lib
@@ -178,6 +180,13 @@ class Oracle:
         if canonical:
             self.sort(ends, pids)
         return ends, pids
+
+    def transitions(self, text):
+        """(goto transitions, failure transitions) of the walk over the text (P6)."""
+        t = _as_u8(text)
+        out = np.zeros(2, dtype=np.uint64)
+        self._lib.oracle_transitions(self._h, _ptr(t, _u8p), t.size, _ptr(out, _u64p))
+        return int(out[0]), int(out[1])
 
     def sort(self, ends: np.ndarray, pids: np.ndarray) -> None:
         """In-place canonical sort (start asc, pid asc) done by the C oracle."""

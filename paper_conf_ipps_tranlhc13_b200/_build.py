@@ -61,7 +61,7 @@ def build(force: bool = False, verbose: bool = False) -> Path:
     with ThreadPoolExecutor(max_workers=max(1, min(8, os.cpu_count() or 1))) as ex:
         objs = list(ex.map(compile_one, sources()))
     tmp = LIB.with_suffix(f".so.tmp{os.getpid()}")
-    subprocess.check_call([nvcc(), *ARCH, "-shared", "-o", str(tmp), *map(str, objs)])
+    subprocess.check_call([nvcc(), *ARCH, "-shared", "-o", str(tmp), *map(str, objs), "-ldl"])  # -ldl: NVTX3
     os.replace(tmp, LIB)
     return LIB
 

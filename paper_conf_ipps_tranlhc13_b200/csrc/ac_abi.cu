@@ -11,6 +11,7 @@
 #include <string>
 
 #include <cudaTypedefs.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "ac_internal.h"
 #include "ac_scan.cuh"
@@ -62,6 +63,14 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
     });
     return fn;
 }
+
+// NVTX range for the scope of a host call (header-only NVTX3: a no-op unless
+// a profiler injects itself), so ncu/nsys timelines show build, scan,
+// gather and host-pipeline phases by name.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 // Makes `device` current for the scope of a call and restores the caller's.
 struct DeviceGuard {
@@ -194,7 +203,11 @@ static SttView view_of(const ac_stt *h, int v) {
     s.stride2 = h->host.stride2;
     s.n_classes = h->host.n_classes;
     s.sblob = nullptr;
+    s.crec = nullptr;
     s.s_dense = s.s_rec = s.s_row_bytes = s.s_rec_x0 = 0;
+    s.stt_evict_last = 0;
+    s.cmap_ident = 1;
+    for (int b = 0; b < 256; b++) s.cmap_ident &= h->host.class_map[b] == b ? 1u : 0u;
     if (h->tier == AC_TIER_SPLIT) {
         // the staged kernel stages the split blob; the global-only kernel
         // (head/tail chains, short texts, re-walks) reads the global table
@@ -202,11 +215,13 @@ static SttView view_of(const ac_stt *h, int v) {
         s.smem_bytes = 0;
         if (v && h->host.split.size() <= stt_budget(h, v)) {
             s.sblob = h->d_split;
+            s.crec = reinterpret_cast<const uint4 *>(h->d_crec);
             s.smem_bytes = (uint32_t)h->host.split.size();
             s.s_dense = h->host.s_dense;
             s.s_rec = h->host.s_rec;
             s.s_row_bytes = 2 * h->host.s_dstride;
-            s.s_rec_x0 = s.s_dense * s.s_row_bytes - 8u * s.s_dense;
+            // records follow the dense rows + escape row; record of id s at s_rec_x0 + 8 s
+            s.s_rec_x0 = (s.s_dense + 1) * s.s_row_bytes - 8u * s.s_dense;
         }
         return s;
     }
@@ -239,6 +254,8 @@ static void free_device(ac_stt *h) {
     h->d_stt2 = nullptr;
     cudaFree(h->d_split);
     h->d_split = nullptr;
+    cudaFree(h->d_crec);
+    h->d_crec = nullptr;
     cudaFree(h->d_class_map);
     cudaFree(h->d_out_off);
     cudaFree(h->d_out_ids);
@@ -252,6 +269,7 @@ static void free_device(ac_stt *h) {
 static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_owned, uint64_t n_halo,
                              uint64_t base, ac_match_t *d_out, uint64_t cap, ac_result *d_res, cudaStream_t stream,
                              const ac_match_opts *opts) {
+    NvtxRange range(d_out ? "ac_match(list)" : "ac_match(count)");
     g_launches = 0;
     g_scratch_rec = 0;
     if (!h || !d_res || (!d_text && n_owned + n_halo > 0)) {
@@ -268,6 +286,10 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         return AC_ERR_TOO_LARGE;
     }
     uint32_t kernel = opts ? opts->kernel : AC_KERNEL_AUTO;
+    if (opts && (opts->text_policy > 2 || opts->stt_policy > 2)) {
+        set_error("text_policy and stt_policy must be 0, 1 or 2");
+        return AC_ERR_INVALID_ARG;
+    }
     if (kernel > AC_KERNEL_GLOBAL) {
         set_error("unknown kernel");
         return AC_ERR_INVALID_ARG;
@@ -310,6 +332,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         return AC_ERR_INVALID_ARG;
     }
     SttView sg = view_of(h, 0), ss = view_of(h, variant);
+    ss.stt_evict_last = opts && opts->stt_policy == 2 ? 1u : 0u;
     // the two-byte walk exists for the two 32-warp x 16-byte shapes only
     if ((opts && opts->stride == 1) || (variant != 4 && variant != 7)) ss.stt2 = nullptr;
     const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
@@ -345,8 +368,10 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             g.n_chains = n_main;
             g.chain0 = ra.n_chains;
             g.n_readable = n_total - head;
+            const uint32_t tp = opts ? opts->text_policy : 0;
             g.text_evict_first =
-                (tier_s == AC_TIER_GLOBAL || tier_s == AC_TIER_HYBRID || tier_s == AC_TIER_SPLIT) ? 1u : 0u;
+                tp ? (tp == 2 ? 1u : 0u)
+                   : (tier_s == AC_TIER_GLOBAL || tier_s == AC_TIER_HYBRID || tier_s == AC_TIER_SPLIT) ? 1u : 0u;
             PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
             if (!enc) {
                 set_error("cuTensorMapEncodeTiled unavailable from the driver");
@@ -647,6 +672,7 @@ static ac_status host_pipe(int device, HostPipe **out) {
 
 static ac_status match_host_pipelined(const ac_stt *stt, const uint8_t *h_text, uint64_t n, ac_match_t *h_out,
                                       uint64_t cap, uint64_t *count, cudaStream_t s) {
+    NvtxRange range("ac_match_host");
     int prev = -1;
     cudaGetDevice(&prev);
     AC_CUDA(cudaSetDevice(stt->device), "cudaSetDevice");
@@ -845,11 +871,14 @@ static void fill_info(const ac_table &t, ac_stt_info *info) {
     info->split_dstride = t.s_dstride;
     info->split_cold_records = t.s_cold_rec;
     info->split_bytes = t.split.size();
+    info->split_cold_full = t.s_cold_full;
+    info->split_crec_bytes = (uint64_t)t.crec.size() * 4;
 }
 
-ac_status ac_table_export_split(const ac_table *t, void *blob) {
+ac_status ac_table_export_split(const ac_table *t, void *blob, uint32_t *crec) {
     if (!t || t->split.empty() || !blob) return AC_ERR_INVALID_ARG;
     std::memcpy(blob, t->split.data(), t->split.size());
+    if (crec) std::memcpy(crec, t->crec.data(), t->crec.size() * 4);
     return AC_OK;
 }
 
@@ -902,6 +931,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
         set_error("unknown tier");
         return AC_ERR_INVALID_ARG;
     }
+    NvtxRange range("ac_build");
     cudaDeviceProp prop;
     ac_status rc = check_device(device, &prop);
     if (rc != AC_OK) return rc;
@@ -1028,6 +1058,9 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             return fail(e, "cudaMalloc(split)");
         if ((e = cudaMemcpy(h->d_split, t.split.data(), t.split.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
             return fail(e, "H2D split");
+        if ((e = cudaMalloc(&h->d_crec, t.crec.size() * 4)) != cudaSuccess) return fail(e, "cudaMalloc(crec)");
+        if ((e = cudaMemcpy(h->d_crec, t.crec.data(), t.crec.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
+            return fail(e, "H2D crec");
     }
     const std::vector<uint8_t> &blob = tier == AC_TIER_COMPACT ? t.compact : t.stt;
     const size_t stt_alloc = (blob.size() + 15) / 16 * 16 + 16;

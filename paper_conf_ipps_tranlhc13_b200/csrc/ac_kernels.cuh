@@ -142,45 +142,82 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
     return sp ? (need ? e3 : ex) : lo;
 }
 
+// SPLIT tier, cold lanes: the state's 16-byte cold record (global, L2
+// resident) -- three exceptions with 32-bit targets over the shared-memory
+// row of fd -- and, for states with more exceptions or an escaped row entry,
+// the full dense table.  The record loads carry an L2 evict-last hint when
+// st.stt_evict_last is set (the instruction-level form of an L2
+// access-policy window over the cold part of the automaton).
+__device__ __forceinline__ uint32_t split_cold(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
+    uint4 r;
+    if (st.stt_evict_last) {
+        uint64_t pol;
+        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+        asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                     : "l"(st.crec + s), "l"(pol));
+    } else {
+        r = __ldg(st.crec + s);
+    }
+    uint32_t row = s;  // full-table row to read if the record cannot answer
+    const uint32_t fd = r.x & 0xFFFFu;
+    if (fd != 0xFFFFu) {
+        const uint32_t x = r.x ^ (cls * 0x01010000u);
+        if ((x & 0x00FF0000u) == 0) return r.y;
+        if (x < 0x01000000u) return r.z;
+        if ((r.w & 0xFFu) == cls) return ((r.w >> 8) & 0x7FFFFFu) | (r.w & 0x80000000u);
+        uint32_t e = base + fd * st.s_row_bytes + cls * 2u;
+        asm("ld.shared.u16 %0, [%0];" : "+r"(e));
+        if (e != 0xFFFFu) return (e >> 1) | (e << 31);
+        row = fd;  // delta(s, cls) = delta(fd, cls), whose 16-bit entry escaped
+    }
+    return __ldg(static_cast<const uint32_t *>(st.stt) + ((size_t)row * st.stride + cls));
+}
+
 // SPLIT tier (ac_split.cpp): delta(s, cls) as a 32-bit entry (BFS id | flag
-// << 31).  Dense rows (s < s_dense) and 8-byte records (s < s_dense + s_rec)
-// are in shared memory; cold states, cold records (fd = 0xFFFF) and escaped
-// 16-bit entries (0xFFFF: next id >= 32767) read the global table through
-// L1/L2.  Every load is predicated, so lanes in different parts of the
-// automaton never diverge; the cold lanes' global load is issued first, in
-// parallel with the shared-memory loads.
+// << 31) by one rule for every hot state: delta = t1 if cls == c1, t2 if
+// cls == c2, else row[fd][cls].  Only sparse hot states (s_dense <= s <
+// s_rec) load their 8-byte record; the others start from (fd = s for a
+// dense state, fd = the all-0xFFFF escape row for a cold one; exception
+// classes ~cls, which never match), so every lane runs the same
+// instructions.  A 16-bit result of 0xFFFF -- cold state, cold record or a
+// next id >= 32767 -- is replaced by the full entry from the global table
+// (L1/L2).
 __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
-    const uint32_t in_d = s < st.s_dense;
-    const uint32_t in_w = (s - st.s_dense) < st.s_rec;
-    const uint32_t cold = (in_d | in_w) ^ 1u;
-    const uint64_t ga = reinterpret_cast<uint64_t>(static_cast<const uint32_t *>(st.stt)) +
-                        ((uint64_t)s * st.stride + cls) * 4u;
-    uint32_t g = 0;
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u32 %0, [%1];\n\t}"
-                 : "+r"(g)
-                 : "l"(ga), "r"(cold));
-    uint32_t lo = base + s * st.s_row_bytes + cls * 2u;  // dense entry (s, cls)
-    uint32_t hi = base + st.s_rec_x0 + s * 8u;           // record of s
-    asm("{\n\t.reg .pred p, q;\n\tsetp.ne.u32 p, %2, 0;\n\tsetp.ne.u32 q, %3, 0;\n\t"
-        "@p ld.shared.v2.u32 {%0, %1}, [%1];\n\t"
-        "@q ld.shared.u16 %0, [%0];\n\t}"
+    const uint32_t sparse = (s - st.s_dense) < (st.s_rec - st.s_dense);
+    uint32_t lo = min(s, st.s_dense) | ((cls ^ 0xFFu) * 0x01010000u);
+    uint32_t hi = base + st.s_rec_x0 + s * 8u;  // record address (biased by -8 s_dense)
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%1];\n\t}"
         : "+r"(lo), "+r"(hi)
-        : "r"(in_w), "r"(in_d));
-    // record: lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
-    const uint32_t fd = lo & 0xFFFFu;
-    const uint32_t h1 = ((lo >> 16) & 0xFFu) == cls, h2 = (lo >> 24) == cls;
-    const uint32_t ovf = in_w & (fd == 0xFFFFu ? 1u : 0u);
-    const uint32_t need = in_w & ((h1 | h2 | ovf) ^ 1u);
-    uint32_t e3 = base + fd * st.s_row_bytes + cls * 2u;  // dense entry (fd, cls)
-    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
-        : "+r"(e3)
-        : "r"(need));
-    const uint32_t e16 = in_d ? lo : h1 ? (hi & 0xFFFFu) : h2 ? (hi >> 16) : e3;
-    const uint32_t esc = (cold ^ 1u) & ((e16 == 0xFFFFu ? 1u : 0u) | ovf);
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.global.nc.u32 %0, [%1];\n\t}"
-                 : "+r"(g)
-                 : "l"(ga), "r"(esc));
-    return (cold | esc) ? g : ((e16 >> 1) | (e16 << 31));
+        : "r"(sparse));
+    // lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
+    const uint32_t x = lo ^ (cls * 0x01010000u);  // c1, c2 bytes become 0 where they match
+    const uint32_t h1 = (x & 0x00FF0000u) == 0, h2 = x < 0x01000000u;
+    uint32_t e = base + (lo & 0xFFFFu) * st.s_row_bytes + cls * 2u;  // row[fd][cls]
+    asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
+        : "+r"(e)
+        : "r"(h1 | h2));
+    const uint32_t e16 = h1 ? (hi & 0xFFFFu) : h2 ? (hi >> 16) : e;
+    uint32_t g = (e16 >> 1) | (e16 << 31);  // 2 x + flag -> x | flag << 31
+    if (e16 == 0xFFFFu) g = split_cold(base, st, s, cls);
+    return g;
+}
+
+// Class of a text byte (a4): the 256-byte class map in shared
+// memory; SPLIT automata whose map is the identity (every byte occurs in a
+// pattern, e.g. C3) skip the load -- one shared-memory wavefront group less
+// per byte.
+template <int TIER>
+__device__ __forceinline__ uint32_t class_of(const uint8_t *s_cmap, uint32_t byte, const SttView &st) {
+    if constexpr (TIER == AC_TIER_SPLIT) {
+        uint32_t c = byte;
+        asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p ld.shared.u8 %0, [%2];\n\t}"
+            : "+r"(c)
+            : "r"(st.cmap_ident), "r"(smem_u32(s_cmap) + byte));
+        return c;
+    } else {
+        return s_cmap[byte];
+    }
 }
 
 // Entry -> next state and output flag.
@@ -214,7 +251,7 @@ __device__ __forceinline__ uint32_t next_entry(const E *s_stt, const SttView &st
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t ac_move(uint32_t s, uint32_t byte, const uint8_t *s_cmap, const E *s_stt,
                                             const SttView &st) {
-    return state_of<E, TIER>(next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]), st);
+    return state_of<E, TIER>(next_entry<E, TIER>(s_stt, st, s, class_of<TIER>(s_cmap, byte, st)), st);
 }
 
 // COMPACT output table slot of output state s: (payload, count).
@@ -361,6 +398,21 @@ __device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t
     }
 }
 
+// emit_outputs out of line, for tiers whose matches are rare (SPLIT): the
+// 16-byte walk loop is unrolled, and inlining the emission at every byte
+// multiplies its code past the instruction cache.  State goes in and out by
+// value so nothing is spilled to the stack.
+struct CntWp {
+    uint32_t cnt;
+    uint64_t wp;
+};
+template <typename E, int TIER, int MODE>
+__device__ __noinline__ CntWp emit_outputs_rare(uint32_t x, uint64_t key0, uint32_t cnt, uint64_t wp, const E *s_stt,
+                                                const SttView &st, const ScanOut &so) {
+    emit_outputs<E, TIER, MODE>(x, key0, cnt, wp, s_stt, st, so);
+    return CntWp{cnt, wp};
+}
+
 // One transition inside the owned chunk: count or emit output(s) at the
 // byte whose record key is key0 = (global start) << 24.  cnt is the chain's
 // running count (32-bit: the planner keeps chain_len x max|output| < 2^31).
@@ -371,7 +423,7 @@ template <typename E, int TIER, int MODE>
 __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp, uint32_t byte, uint64_t key0,
                                         bool live, const uint8_t *s_cmap, const E *s_stt, const SttView &st,
                                         const ScanOut &so) {
-    const uint32_t e = next_entry<E, TIER>(s_stt, st, s, s_cmap[byte]);
+    const uint32_t e = next_entry<E, TIER>(s_stt, st, s, class_of<TIER>(s_cmap, byte, st));
     s = state_of<E, TIER>(e, st);
     const uint32_t flag = flag_of<E, TIER>(e, s, st);
     // Predication pays where matches are dense (C2-like dictionaries, which are
@@ -1011,6 +1063,30 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                                                     kb[k] + ((uint64_t)bb << 24), kb[k] + ((uint64_t)(bb - 1) << 24),
                                                     live[k], s_cmap, s_stt, st, so);
                     }
+                } else if constexpr (TIER == AC_TIER_SPLIT) {
+                    // rare matches (the tier is chosen for large byte
+                    // dictionaries): the walk is the whole loop body; the
+                    // record key and the chain's liveness are only touched
+                    // on a flagged byte
+#pragma unroll
+                    for (int bb = 15; bb >= 0; --bb) {
+#pragma unroll
+                        for (int k = 0; k < K; k++) {
+                            const uint32_t e =
+                                next_entry<E, TIER>(s_stt, st, s[k], class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                            s[k] = state_of<E, TIER>(e, st);
+                            if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k]) {
+                                if constexpr (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT) {
+                                    const CntWp r = emit_outputs_rare<E, TIER, MODE>(
+                                        s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt, st, so);
+                                    cnt[k] = r.cnt;
+                                    wp[k] = r.wp;
+                                } else {
+                                    cnt[k] += out_count<E, TIER>(s_stt, st, s[k]);
+                                }
+                            }
+                        }
+                    }
                 } else {
 #pragma unroll
                     for (int bb = 15; bb >= 0; --bb) {
@@ -1201,8 +1277,7 @@ cudaError_t launch_staged_tier(int mode, uint32_t eb, int variant, const CUtenso
             return launch_staged_m<uint32_t, TIER, decltype(m)::value>(variant, tmap, mtext, st, g, so, smem_stt,
                                                                        stream);
         });
-    }
-    if (eb == 2)
+    } else if (eb == 2)
         return with_mode(mode, [&](auto m) {
             return launch_staged_m<uint16_t, TIER, decltype(m)::value>(variant, tmap, mtext, st, g, so, smem_stt,
                                                                        stream);

@@ -41,11 +41,15 @@ struct SttView {
     const uint32_t *stt2;
     uint32_t stride2, n_classes;
     // SPLIT tier (ac_split.cpp): shared-memory part staged from `sblob` --
-    // dense rows of BFS ids [0, s_dense) at s * s_row_bytes, 8-byte records
-    // of ids [s_dense, s_dense + s_rec) at s_rec_x0 + 8 s (biased, wraps);
+    // dense rows r <= s_dense at r * s_row_bytes (row s_dense = the escape
+    // row), the 8-byte records of the sparse hot ids [s_dense, s_rec) at
+    // s_rec_x0 + 8 s (biased by -8 s_dense, wraps);
     // `stt` stays the full 32-bit table for the cold states
     const void *sblob;
+    const uint4 *crec;  // cold records (global, 16 B per state)
     uint32_t s_dense, s_rec, s_row_bytes, s_rec_x0;
+    uint32_t cmap_ident;  // the class map is the identity (every byte occurs in a pattern)
+    uint32_t stt_evict_last;  // SPLIT: cold global-table loads carry an L2 evict-last hint
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.

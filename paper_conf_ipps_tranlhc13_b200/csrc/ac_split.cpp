@@ -12,24 +12,37 @@
 // on the C3 text: depth 1 = 60 %, depth 2 = 38 %, deeper 2 %), and in the AC
 // automaton delta(s,c) = g(s,c) if the trie has that edge, else
 // delta(f(s),c) (P:62 with the failure function of P:52).  So, in BFS order
-// (states sorted by depth, the ids of the global dense table):
+// (states sorted by depth, the ids of the global dense table), the HOT
+// states [0, H) are served from shared memory by one rule:
 //
-//   * ids [0, D)      DENSE rows in shared memory: C 16-bit entries each;
-//   * ids [D, D + W)  8-byte RECORDS in shared memory: fd(s) = the first
-//                     dense state on s's failure chain and two exceptions
-//                     (c, delta(s,c)) -- the classes where delta(s,.)
-//                     differs from delta(fd(s),.); states needing more are
-//                     marked cold (fd = 0xFFFF);
-//   * everything else COLD: the full dense 32-bit table in global memory,
-//                     read through L1/L2.
+//   record(s) = fd(s) | c1 << 16 | c2 << 24,  t1 | t2 << 16
+//   delta(s, c) = t1 if c == c1, t2 if c == c2, else row[fd(s)][c]
 //
-// A shared-memory entry is 2 x + flag (x = BFS id of the next state, flag =
-// output(x) != {}) when x < 32767, else 0xFFFF = "read this entry from the
-// global table".  Records with fewer than two exceptions repeat a real one
-// (or store delta(s, 0)) so no sentinel class is needed: every stored
-// (c, t) pair is exactly delta(s, c).  Output enumeration always reads the
-// global table's per-row output summary (matches are rare where this tier
-// is chosen).
+// where row[] are dense 16-bit rows, also in shared memory:
+//   * the shallow levels [0, D) are DENSE: no record is stored; the kernel
+//     uses (fd = s, no exception class), i.e. reads the state's own row;
+//   * the next states [D, H) are SPARSE: fd(s) = the first dense state on s's
+//     failure chain, (c1, t1), (c2, t2) = the (at most two) classes where
+//     delta(s,.) differs from delta(fd(s),.) -- repeated, or (0, delta(s, 0)),
+//     when there are fewer, so every stored pair is exactly delta(s, c);
+//   * a sparse state needing more exceptions is COLD: its record points at
+//     row[D], the ESCAPE row (all 0xFFFF), with t1 = t2 = 0xFFFF;
+//   * states >= H are COLD: the kernel does not read a record for them.
+// A 16-bit entry is 2 x + flag (x = BFS id of the next state, flag =
+// output(x) != {}) when x < 32767, else 0xFFFF; 0xFFFF (cold state, cold
+// record, large id) sends the lane to global memory:
+//   * first the COLD RECORD of s, 16 bytes per state (2 MB for C3, so it
+//     stays L2-resident next to the streamed text):
+//       w0 = fd | c1 << 16 | c2 << 24, w1 = t1, w2 = t2, w3 = c3 | t3 << 8
+//     the same rule with three exceptions and 32-bit (24-bit for t3)
+//     entries, fd = the first dense state on s's failure chain (whose row is
+//     in shared memory);
+//   * states needing more exceptions (fd = 0xFFFF), and dense-row entries
+//     that escaped, read the full 32-bit dense table (the paper's STT,
+//     P:118) -- 137 MB for C3, mostly DRAM-resident, now touched by < 1 % of
+//     the steps.
+// Output enumeration always reads that table's per-row output summary
+// (matches are rare where this tier is chosen).
 #include <algorithm>
 #include <cstring>
 
@@ -81,42 +94,70 @@ bool split_table(ac_table &t, size_t budget) {
         D = hi;
     }
     if ((size_t)D * row_bytes > budget || D >= 0xFFFFu) return false;
-    const size_t dense_bytes = (size_t)D * row_bytes;
-    const uint32_t W = (uint32_t)std::min<size_t>(S - D, (budget - dense_bytes) / 8);
+    const size_t dense_bytes = (size_t)(D + 1) * row_bytes;  // + the escape row
+    if (dense_bytes > budget) return false;
+    const uint32_t H = D + (uint32_t)std::min<size_t>(S - D, (budget - dense_bytes) / 8);
     set_fd(D);
 
     auto enc = [&](uint32_t e) -> uint16_t {  // 32-bit entry -> 2 x + flag, or the escape
         const uint32_t x = e & 0x7fffffffu;
         return x < 32767u ? (uint16_t)((x << 1) | (e >> 31)) : (uint16_t)0xFFFFu;
     };
-    std::vector<uint8_t> blob(dense_bytes + (size_t)W * 8, 0);
+    std::vector<uint8_t> blob(dense_bytes + (size_t)(H - D) * 8, 0);
     for (uint32_t s = 0; s < D; s++)
         for (uint32_t c = 0; c < C; c++) {
             const uint16_t e = enc(delta(s, c));
             std::memcpy(&blob[((size_t)s * dstride + c) * 2], &e, 2);
         }
+    for (uint32_t c = 0; c < dstride; c++) {  // the escape row
+        const uint16_t e = 0xFFFFu;
+        std::memcpy(&blob[((size_t)D * dstride + c) * 2], &e, 2);
+    }
     uint32_t n_cold = 0;
-    for (uint32_t i = 0; i < W; i++) {
-        const uint32_t s = D + i;
-        uint32_t cls[2] = {0, 0};
-        const uint32_t k = exceptions(s, fd[s], cls, 2);
-        uint32_t lo, hi;
-        if (k > 2) {  // cold record: the global table serves this state
-            lo = 0xFFFFu;
-            hi = 0;
-            n_cold++;
-        } else {
-            if (k == 1) cls[1] = cls[0];
-            // k == 0: (0, delta(s, 0)) twice -- equal to the dense fallback anyway
-            lo = fd[s] | (cls[0] << 16) | (cls[1] << 24);
-            hi = (uint32_t)enc(delta(s, cls[0])) | ((uint32_t)enc(delta(s, cls[1])) << 16);
+    for (uint32_t s = D; s < H; s++) {  // records of the sparse hot states
+        uint32_t cls[2] = {0, 0}, lo, hi;
+        {
+            const uint32_t k = exceptions(s, fd[s], cls, 2);
+            if (k > 2) {  // cold record: every class escapes to the global table
+                lo = D;
+                hi = 0xFFFFFFFFu;
+                n_cold++;
+            } else {
+                if (k == 1) cls[1] = cls[0];
+                // k == 0: (0, delta(s, 0)) twice -- equal to the dense fallback anyway
+                lo = fd[s] | (cls[0] << 16) | (cls[1] << 24);
+                hi = (uint32_t)enc(delta(s, cls[0])) | ((uint32_t)enc(delta(s, cls[1])) << 16);
+            }
         }
-        std::memcpy(&blob[dense_bytes + (size_t)i * 8], &lo, 4);
-        std::memcpy(&blob[dense_bytes + (size_t)i * 8 + 4], &hi, 4);
+        std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8], &lo, 4);
+        std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8 + 4], &hi, 4);
+    }
+    // cold records of every state (dense states: marker, never used)
+    std::vector<uint32_t> crec((size_t)S * 4, 0);
+    uint32_t n_cold_full = 0;
+    for (uint32_t s = 0; s < S; s++) {
+        uint32_t *r = &crec[(size_t)s * 4];
+        uint32_t cls[3] = {0, 0, 0};
+        const uint32_t k = s < D ? 4u : exceptions(s, fd[s], cls, 3);
+        if (k == 0) cls[0] = 0;
+        if (k <= 1) cls[1] = cls[0];
+        if (k <= 2) cls[2] = cls[1];
+        const uint32_t t3 = delta(s, cls[2]);
+        if (k > 3 || (t3 & 0x7fffffffu) >= (1u << 23)) {
+            r[0] = 0xFFFFu;  // read the dense global row
+            n_cold_full += s >= D;
+            continue;
+        }
+        r[0] = fd[s] | (cls[0] << 16) | (cls[1] << 24);
+        r[1] = delta(s, cls[0]);
+        r[2] = delta(s, cls[1]);
+        r[3] = cls[2] | ((t3 & 0x7fffffu) << 8) | ((t3 >> 31) << 31);
     }
     t.split.swap(blob);
+    t.crec.swap(crec);
+    t.s_cold_full = n_cold_full;
     t.s_dense = D;
-    t.s_rec = W;
+    t.s_rec = H;
     t.s_dstride = dstride;
     t.s_cold_rec = n_cold;
     return true;

@@ -1,0 +1,76 @@
+"""Tier experiment on one GPU: count-mode scan time of the staged kernel for
+several dictionaries and STT tiers (development tool; bench.py is the
+contract).  One JSON line per (workload, tier, variant)."""
+from __future__ import annotations
+
+import argparse
+import json
+import sys
+from pathlib import Path
+
+ROOT = Path(__file__).resolve().parents[1]
+sys.path.insert(0, str(ROOT))
+
+import torch  # noqa: E402
+
+import paper_conf_ipps_tranlhc13_b200 as ac  # noqa: E402
+import synth  # noqa: E402
+
+TIERS = {"auto": ac.TIER_AUTO, "global": ac.TIER_GLOBAL, "split": ac.TIER_SPLIT, "compact": ac.TIER_COMPACT}
+
+
+def timeit(fn, reps=10, warm=3):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(reps):
+        fn()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / reps
+
+
+def main():
+    p = argparse.ArgumentParser()
+    p.add_argument("--workloads", default="c3")
+    p.add_argument("--n", type=int, default=1 << 28)
+    p.add_argument("--tiers", default="global,split")
+    p.add_argument("--variants", default="0")
+    p.add_argument("--list", action="store_true")
+    p.add_argument("--policies", default="0", help="text L2 policies (0 auto, 1 evict-normal, 2 evict-first)")
+    a = p.parse_args()
+    for name in a.workloads.split(","):
+        w = synth.make(name, n=a.n)
+        n = w.text.size
+        text = torch.from_numpy(w.text).cuda()
+        res = torch.zeros(2, dtype=torch.int64, device="cuda")
+        for tname in a.tiers.split(","):
+            try:
+                stt = ac.build(w.patterns, tier=TIERS[tname])
+            except ac.AcError as e:
+                print(json.dumps({"workload": name, "tier": tname, "skipped": str(e)}), flush=True)
+                continue
+            out = torch.empty(n // 8 + 64, dtype=torch.int64, device="cuda") if a.list else None
+            for v, pol in [(v, pol) for v in a.variants.split(",") for pol in a.policies.split(",")]:
+                tpol, spol = (pol + ":0").split(":")[:2]  # text policy[:stt policy]
+                knobs = dict(kernel=ac.KERNEL_STAGED, variant=int(v), text_policy=int(tpol), stt_policy=int(spol))
+                try:
+                    ac.match_async(stt, text, out, res, **knobs)
+                except ac.AcError as e:
+                    print(json.dumps({"workload": name, "tier": tname, "variant": v, "skipped": str(e)}), flush=True)
+                    continue
+                t = timeit(lambda: ac.match_async(stt, text, out, res, **knobs))
+                print(json.dumps({"workload": name, "n": n, "tier": stt.tier_name, "variant": int(v),
+                                  "policy": pol, "list": bool(a.list),
+                                  "states": stt.info["n_states"], "split_dense": stt.info["split_dense"],
+                                  "split_records": stt.info["split_records"], "ms": round(t, 4),
+                                  "gbps": round(n * 8 / t / 1e6, 1), "matches": int(res[0]),
+                                  "names": ac.last_launch_names()}), flush=True)
+            del stt
+        del text
+
+
+if __name__ == "__main__":
+    main()

@@ -2,11 +2,12 @@
 English-like (C2) and Snort-like (C3) families, plus the high-match-rate adversarial texts.
 One JSON line per point: count and list Gbps (CUDA events, text resident, STT built),
 tier, states, matches, and a parity verdict against the CPU oracle (test infrastructure,
-oracle/) on sampled windows -- or the closed form K*n - K(K-1)/2 for a^n with {a^1..a^K}
-(SURVEY 8(c) P4-i), whose list does not fit in memory.  Development tool, like sweep.py;
-bench.py is the contract.
+oracle/): the full count plus the multiset digest of the whole list (oracle windows on every
+host core) up to --digest-max bytes of text, sampled windows beyond -- or the closed form
+K*n - K(K-1)/2 for a^n with {a^1..a^K}, whose list does not fit in memory.
+Development tool, like sweep.py; bench.py is the contract.
 
-    python scripts/sweep_c5.py [--logn 26,28] [--patterns 1000,5000,20000,50000]
+    python scripts/sweep_c5.py [--logn 26,28,30] [--patterns 1000,5000,10000,20000,50000]
 """
 from __future__ import annotations
 
@@ -25,6 +26,11 @@ import torch  # noqa: E402
 import paper_conf_ipps_tranlhc13_b200 as ac  # noqa: E402
 import synth  # noqa: E402
 from oracle import Oracle  # noqa: E402
+
+sys.path.insert(0, str(ROOT / "tests"))
+from test_gpu_parity import digest_keys  # noqa: E402
+
+DIGEST_MAX = 1 << 30
 
 
 def timeit(fn, reps=5, warm=2):
@@ -74,7 +80,12 @@ def point(label, pats, text_np, list_budget=12 << 30, closed_form=None):
         assert int(res[0]) == cnt and int(res[1]) == 0
         line.update(list_ms=round(t_list, 4), list_gbps=round(n * 8 / t_list / 1e6, 1))
         recs = out[:cnt].cpu().numpy()
-        line["parity"] = ("oracle windows: ok" if windows_ok(pats, text_np, recs) else "oracle windows: MISMATCH")
+        if n <= DIGEST_MAX:
+            t0 = time.time()
+            ok = digest_keys(recs) == Oracle(pats).digest_parallel(text_np)
+            line["parity"] = f"whole-text count + digest ({time.time() - t0:.0f} s): " + ("ok" if ok else "MISMATCH")
+        else:
+            line["parity"] = ("oracle windows: ok" if windows_ok(pats, text_np, recs) else "oracle windows: MISMATCH")
         del out
     else:
         line["list"] = f"skipped: {cnt} records > list budget"
@@ -90,7 +101,9 @@ def main():
     p.add_argument("--logn", default="26,28")
     p.add_argument("--patterns", default="1000,5000,20000,50000")
     p.add_argument("--families", default="english,snort,adv")
+    p.add_argument("--digest-max", type=int, default=DIGEST_MAX)
     a = p.parse_args()
+    globals()["DIGEST_MAX"] = a.digest_max
     Ps = [int(x) for x in a.patterns.split(",")]
     fams = a.families.split(",")
     for logn in [int(x) for x in a.logn.split(",")]:

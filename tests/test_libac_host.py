@@ -274,27 +274,28 @@ def test_compact_rejects_wide_alphabets():
 
 
 def _decode_split(t):
-    """The SPLIT lookup rule of include/ac.h, vectorised over the states in
-    shared memory: E[s, c] = 32-bit entry (BFS id | flag << 31) where the
-    shared-memory part answers, -1 where the global table must (cold record or
-    escaped entry)."""
+    """The SPLIT lookup rule of include/ac.h, vectorised over the hot states:
+    E[s, c] = 32-bit entry (BFS id | flag << 31) where the shared-memory part
+    answers, -1 where the global table must (cold record or escaped entry)."""
     d = t.info
     C = d["n_classes"]
-    D, W, ds = d["split_dense"], d["split_records"], d["split_dstride"]
+    D, H, ds = d["split_dense"], d["split_records"], d["split_dstride"]
     blob = t.split
-    dense = blob[:D * ds * 2].view(np.uint16).reshape(D, ds)[:, :C].astype(np.int64)
-    rec = blob[D * ds * 2:D * ds * 2 + W * 8].view(np.uint32).reshape(-1, 2).astype(np.int64)
-    fd = rec[:, 0] & 0xFFFF
-    c1, c2 = (rec[:, 0] >> 16) & 0xFF, rec[:, 0] >> 24
-    t1, t2 = rec[:, 1] & 0xFFFF, rec[:, 1] >> 16
+    rows = blob[:(D + 1) * ds * 2].view(np.uint16).reshape(D + 1, ds)[:, :C].astype(np.int64)
+    assert (rows[D] == 0xFFFF).all()  # the escape row
+    assert blob.size == (D + 1) * ds * 2 + (H - D) * 8
+    rec = blob[(D + 1) * ds * 2:].view(np.uint32).reshape(-1, 2).astype(np.int64)
+    fd = np.concatenate([np.arange(D), rec[:, 0] & 0xFFFF])  # dense states read their own row
+    no = np.full(D, 0x1FF)  # no exception class
+    c1 = np.concatenate([no, (rec[:, 0] >> 16) & 0xFF])
+    c2 = np.concatenate([no, rec[:, 0] >> 24])
+    t1 = np.concatenate([np.zeros(D, np.int64), rec[:, 1] & 0xFFFF])
+    t2 = np.concatenate([np.zeros(D, np.int64), rec[:, 1] >> 16])
+    assert (fd[D:] <= D).all()
     cls = np.arange(C)[None, :]
-    cold = fd == 0xFFFF
-    fb = dense[np.where(cold, 0, fd)]
-    sparse = np.where(cls == c1[:, None], t1[:, None], np.where(cls == c2[:, None], t2[:, None], fb))
-    sparse[cold] = 0xFFFF
-    e16 = np.concatenate([dense, sparse])
+    e16 = np.where(cls == c1[:, None], t1[:, None], np.where(cls == c2[:, None], t2[:, None], rows[fd]))
     E = (e16 >> 1) | ((e16 & 1) << 31)
-    return np.where(e16 == 0xFFFF, -1, E), int(cold.sum())
+    return np.where(e16 == 0xFFFF, -1, E), int((fd[D:] == D).sum())
 
 
 @pytest.mark.parametrize("which", ["c3", "english5k", "tiny"])
@@ -311,10 +312,10 @@ def test_split_encoding_equals_dense(which):
     t = ac.compile_table(pats, split=True)
     d = t.info
     assert d["entry_bytes"] == 4 and d["split_bytes"] > 0
-    C, D, W = d["n_classes"], d["split_dense"], d["split_records"]
+    C, D, H = d["n_classes"], d["split_dense"], d["split_records"]
     E, n_cold = _decode_split(t)
     assert n_cold == d["split_cold_records"]
-    want = t.stt[:D + W, :C].astype(np.int64)
+    want = t.stt[:H, :C].astype(np.int64)
     ok = E >= 0
     assert np.array_equal(E[ok], want[ok])
     # escapes only where the next id does not fit 15 bits, or cold records
@@ -323,7 +324,34 @@ def test_split_encoding_equals_dense(which):
     assert D >= 1
     # fits next to the lean staged variant's ring
     assert d["split_bytes"] <= 232448 - (32 * 2 * 512 + 512 + 16 + 256) - 128
+    # cold records (global): the same rule with three exceptions and 32-bit
+    # targets over the dense rows; fd = 0xFFFF defers to the full table
+    S = d["n_states"]
+    cr = t.crec.astype(np.int64)
+    assert cr.shape == (S, 4) and d["split_crec_bytes"] == 16 * S
+    D1 = d["split_dstride"]
+    rows = t.split[:(D + 1) * D1 * 2].view(np.uint16).reshape(D + 1, D1)[:, :C].astype(np.int64)
+    fd = cr[:, 0] & 0xFFFF
+    ok = fd != 0xFFFF
+    assert not ok[:D].any() and int((~ok[D:]).sum()) == d["split_cold_full"]
+    c1, c2, c3 = (cr[:, 0] >> 16) & 0xFF, cr[:, 0] >> 24, cr[:, 3] & 0xFF
+    t3 = ((cr[:, 3] >> 8) & 0x7FFFFF) | (cr[:, 3] & 0x80000000)
+    rowv = rows[np.where(ok, fd, 0)]
+    rowe = np.where(rowv == 0xFFFF, -1, (rowv >> 1) | ((rowv & 1) << 31))
+    cls = np.arange(C)[None, :]
+    got = np.where(cls == c1[:, None], cr[:, 1:2], np.where(cls == c2[:, None], cr[:, 2:3],
+                   np.where(cls == c3[:, None], t3[:, None], rowe)))
+    full = t.stt[:, :C].astype(np.int64)
+    sel = ok[:, None] & (got >= 0)
+    assert np.array_equal(got[sel], np.broadcast_to(full, got.shape)[sel])
+    # escaped row entries: delta(s, c) = delta(fd, c) (the kernel reads row fd of the full table)
+    esc = ok[:, None] & (got < 0)
+    if esc.any():
+        ss, cc = np.nonzero(esc)
+        assert np.array_equal(full[ss, cc], full[fd[ss], cc])
+    if which == "c3":
+        assert d["split_cold_full"] < S // 20
     if which == "c3":
         # depth <= 1 dense (root + one state per used last byte), depth-2 states as records
         assert D == 1 + len({p[-1] for p in pats})
-        assert W >= 7000 and d["split_cold_records"] < W // 10
+        assert H - D >= 7000 and d["split_cold_records"] < (H - D) // 10

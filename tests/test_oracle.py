@@ -366,3 +366,36 @@ def test_canonical_sort_is_reentrant():
 
     with ThreadPoolExecutor(8) as ex:
         assert all(ex.map(run, cases * 2))
+
+
+# ---------------------------------------------------------------------------
+# P6: the walk is O(n): one goto transition per symbol, and at most as
+# many failure transitions (AC'75: each failure move lowers the depth, each
+# goto move raises it by at most one)
+# ---------------------------------------------------------------------------
+def test_transitions_worked_example():
+    # "ushers": g(5,'r') = fail -> f(5) = 2 is the only failure move
+    o = Oracle([b"he", b"she", b"his", b"hers"])
+    assert o.transitions(b"ushers") == (6, 1)
+
+
+@pytest.mark.parametrize("seed", range(80))
+def test_transitions_linear(seed):
+    rng = random.Random(31000 + seed)
+    A = rng.randint(1, 4)
+    alphabet = list(range(97, 97 + A))
+    pats = [bytes(rng.choice(alphabet) for _ in range(rng.randint(1, 7))) for _ in range(rng.randint(1, 9))]
+    text = bytes(rng.choice(alphabet) for _ in range(rng.randint(0, 500)))
+    o = Oracle(pats)
+    gotos, fails = o.transitions(text)
+    assert gotos == len(text) and fails <= gotos
+
+
+def test_transitions_closed_forms():
+    # a^n with {a^1..a^K}: the walk climbs to depth K, then every further 'a'
+    # is one failure move (a^K -> a^(K-1)) and one goto move: n - K failures
+    K, n = 5, 1000
+    o = Oracle([b"a" * k for k in range(1, K + 1)])
+    assert o.transitions(b"a" * n) == (n, n - K)
+    # no pattern byte in the text: the root loops, no failure move
+    assert Oracle([b"xyz"]).transitions(b"abc" * 50) == (150, 0)
