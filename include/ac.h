@@ -158,13 +158,6 @@ typedef struct {
      * table. */
     uint32_t split_dense, split_records, split_dstride, split_cold_records;
     uint64_t split_bytes;
-    /* SPLIT cold records (global memory, split_crec_bytes = 16 x n_states):
-     * w0 = fd | c1 << 16 | c2 << 24, w1 = t1, w2 = t2 (32-bit entries),
-     * w3 = c3 | t3 << 8 (23-bit id, flag in bit 31); fd = 0xFFFF (the
-     * split_cold_full states needing more exceptions, and the dense states)
-     * = read the 32-bit dense table. */
-    uint32_t split_cold_full, reserved2;
-    uint64_t split_crec_bytes;
 } ac_stt_info;
 
 /* Scan variants (SURVEY 8(f) NEXT-1 ablations are selectable here). */
@@ -182,7 +175,7 @@ typedef struct {
     uint32_t kernel;       /* AC_KERNEL_*                                    */
     uint32_t chain_bytes;  /* bytes owned per thread chain (0 = auto; STAGED:
                               rounded to the tile width)                     */
-    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..7 (DESIGN.md
+    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..10 (DESIGN.md
                               "Staged variants": warps x chains/lane x tile
                               width x ring depth)                            */
     uint32_t scratch_slots;/* list mode: records each chain may park in its
@@ -209,10 +202,12 @@ typedef struct {
     uint32_t text_policy;  /* L2 policy of the staged kernel's text loads:
                               0 = auto (evict-first where the table lives in
                               L2: GLOBAL, HYBRID, SPLIT), 1 = evict-normal,
-                              2 = evict-first (ablation knob)               */
-    uint32_t stt_policy;   /* SPLIT tier: L2 policy of the cold global-table
-                              loads: 0 = auto, 1 = evict-normal, 2 =
-                              evict-last (keeps cold rows ahead of the text) */
+                              2 = evict-first, 3 = per 32-byte sector: the
+                              half read first evict-normal, the second
+                              evict-first (ablation knob)                   */
+    uint32_t text_promotion; /* L2 promotion of the text's TMA misses:
+                              0 = auto (256 B), 1 = none, 2 = 64 B,
+                              3 = 128 B, 4 = 256 B (ablation knob)          */
 } ac_match_opts;
 
 /* Per-call device result written by the async entry points. */
@@ -325,9 +320,8 @@ ac_status ac_table_export_compact(const ac_table *t, void *blob, uint32_t *perm)
  * output(final) != {} | bit 30 = output(middle) != {}. */
 ac_status ac_table_export_stride2(const ac_table *t, uint32_t *tab);
 /* opts->tier == AC_TIER_SPLIT (ac_compile) builds the SPLIT shared-memory
- * part for the default budget (32-bit table); copies its split_bytes and,
- * if crec != NULL, the split_crec_bytes of cold records. */
-ac_status ac_table_export_split(const ac_table *t, void *blob, uint32_t *crec);
+ * part for the default budget (32-bit table); copies its split_bytes. */
+ac_status ac_table_export_split(const ac_table *t, void *blob);
 void ac_table_free(ac_table *t);
 
 /* ------------------------------------------------------------ diagnostics */

@@ -66,8 +66,7 @@ class ac_stt_info(ctypes.Structure):
                 ("stride", ctypes.c_uint32), ("stride2_cols", ctypes.c_uint32), ("stt2_bytes", ctypes.c_uint64),
                 ("split_dense", ctypes.c_uint32), ("split_records", ctypes.c_uint32),
                 ("split_dstride", ctypes.c_uint32), ("split_cold_records", ctypes.c_uint32),
-                ("split_bytes", ctypes.c_uint64), ("split_cold_full", ctypes.c_uint32),
-                ("reserved2", ctypes.c_uint32), ("split_crec_bytes", ctypes.c_uint64)]
+                ("split_bytes", ctypes.c_uint64)]
 
 
 class ac_match_opts(ctypes.Structure):
@@ -76,7 +75,7 @@ class ac_match_opts(ctypes.Structure):
                 ("stride", ctypes.c_uint32),
                 ("n_events", ctypes.c_uint32),
                 ("events", ctypes.POINTER(ctypes.c_void_p)),
-                ("text_policy", ctypes.c_uint32), ("stt_policy", ctypes.c_uint32)]
+                ("text_policy", ctypes.c_uint32), ("text_promotion", ctypes.c_uint32)]
 
 
 _lib = None
@@ -102,7 +101,7 @@ def lib():
         L.ac_table_export.argtypes = [_vp, _vp, _vp, _vp, _vp]
         L.ac_table_export_compact.argtypes = [_vp, _vp, _vp]
         L.ac_table_export_stride2.argtypes = [_vp, _vp]
-        L.ac_table_export_split.argtypes = [_vp, _vp, _vp]
+        L.ac_table_export_split.argtypes = [_vp, _vp]
         L.ac_stt_pattern_lengths.argtypes = [_vp, _vp]
         L.ac_match.argtypes = [_vp, _vp, _u64, _vp, _u64, _u64p, _vp]
         L.ac_match_shard.argtypes = [_vp, _vp, _u64, _u64, _u64, _vp, _u64, _u64p, _vp]
@@ -210,9 +209,9 @@ def _check_text(text: torch.Tensor):
 
 
 def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, scratch_slots: int = 0,
-           two_pass: bool = False, events=None, stride: int = 0, text_policy: int = 0, stt_policy: int = 0):
+           two_pass: bool = False, events=None, stride: int = 0, text_policy: int = 0, text_promotion: int = 0):
     o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, scratch_slots,
-                      int(two_pass), stride, 0, None, text_policy, stt_policy)
+                      int(two_pass), stride, 0, None, text_policy, text_promotion)
     if events:
         arr = (ctypes.c_void_p * (2 * len(events)))(*[e.cuda_event for pair in events for e in pair])
         o.n_events = len(events)
@@ -224,7 +223,7 @@ def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, sc
 def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: torch.Tensor, *,
                 n_halo: int = 0, base: int = 0, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0,
                 variant: int = 0, scratch_slots: int = 0, two_pass: bool = False, stride: int = 0,
-                events=None, text_policy: int = 0, stt_policy: int = 0) -> int:
+                events=None, text_policy: int = 0, text_promotion: int = 0) -> int:
     """Enqueue the scan; result (int64[2] CUDA) receives (count, status).
     ``text`` holds n_owned + n_halo bytes.  ``kernel``/``chain_bytes``/
     ``variant``/``scratch_slots``/``two_pass`` select the scan (ac_match_opts).  ``events``: optional list
@@ -245,7 +244,7 @@ def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: 
         cap = out.numel()
         # non-NULL selects list mode; with cap == 0 the status gates every write
         optr = out.data_ptr() if cap else result.data_ptr()
-    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events, stride, text_policy, stt_policy)
+    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events, stride, text_policy, text_promotion)
     L = lib()
     _check(L.ac_match_async(stt.handle, text.data_ptr() if n_total else None, n_total - n_halo, n_halo, base,
                             optr, cap, result.data_ptr(), _stream_ptr(stream), ctypes.byref(o)))
@@ -369,7 +368,6 @@ class HostTable:
     stt2: "object" = None      # two-byte table (uint32, S x stride2_cols) if requested
     perm: "object" = None      # compact id -> dense BFS id
     split: "object" = None     # SPLIT shared-memory part (uint8) if requested
-    crec: "object" = None      # SPLIT cold records (uint32, S x 4) if requested
 
 
 def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact: bool = False,
@@ -402,13 +400,11 @@ def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact
             t2 = np.zeros(d["n_states"] * d["stride2_cols"], dtype=np.uint32)
             _check(L.ac_table_export_stride2(h, t2.ctypes.data))
             t2 = t2.reshape(d["n_states"], d["stride2_cols"])
-        sp = crec = None
+        sp = None
         if split:
             sp = np.zeros(d["split_bytes"], dtype=np.uint8)
-            crec = np.zeros(d["split_crec_bytes"] // 4, dtype=np.uint32)
-            _check(L.ac_table_export_split(h, sp.ctypes.data, crec.ctypes.data))
-            crec = crec.reshape(-1, 4)
+            _check(L.ac_table_export_split(h, sp.ctypes.data))
         return HostTable(d, cm, stt.reshape(d["n_states"], d["row_stride"]), off, ids[:d["out_entries"]],
-                         compact=blob, stt2=t2, perm=perm, split=sp, crec=crec)
+                         compact=blob, stt2=t2, perm=perm, split=sp)
     finally:
         L.ac_table_free(h)

@@ -40,9 +40,17 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
 static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
 static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)
 static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slots (32 KB ring)
+// SPLIT automata are sized for variant 10 (32 warps x 1 chain, 32-byte tiles,
+// 1 slot refilled as soon as it is copied to registers: 32 KB ring + 1 KB
+// swizzle alignment) so that both it and the lean variant 7 can stage them;
+// AUTO runs variant 7 (C3 list 1.04 vs 1.10 ms per 256 MiB; variant 10 reads
+// every text sector once -- 1.44 vs 3.3 GB of DRAM reads per GiB -- but is
+// not faster: the SPLIT scan is bound by issue and latency, not DRAM)
+static const int kSplitVariant = 10;
 // COMPACT budget used by ac_compile (no device): B200's 227 KB opt-in shared
 // memory minus the lean staged variant's ring and bookkeeping (= stt_budget)
 #define kDefaultCompactBudget (232448 - staged_smem_bytes(staged_variant(kLeanVariant), 0) - 128)
+#define kDefaultSplitBudget (232448 - staged_smem_bytes(staged_variant(kSplitVariant), 0) - 128)
 // Below ~32 MiB the staged kernel cannot fill 148 SMs x 1024 chains with
 // chains of >= 256 B; the global kernel's shorter chains win (C1: 1 MiB list
 // 0.037 ms global vs 0.052 ms staged).
@@ -203,9 +211,7 @@ static SttView view_of(const ac_stt *h, int v) {
     s.stride2 = h->host.stride2;
     s.n_classes = h->host.n_classes;
     s.sblob = nullptr;
-    s.crec = nullptr;
     s.s_dense = s.s_rec = s.s_row_bytes = s.s_rec_x0 = 0;
-    s.stt_evict_last = 0;
     s.cmap_ident = 1;
     for (int b = 0; b < 256; b++) s.cmap_ident &= h->host.class_map[b] == b ? 1u : 0u;
     if (h->tier == AC_TIER_SPLIT) {
@@ -215,7 +221,6 @@ static SttView view_of(const ac_stt *h, int v) {
         s.smem_bytes = 0;
         if (v && h->host.split.size() <= stt_budget(h, v)) {
             s.sblob = h->d_split;
-            s.crec = reinterpret_cast<const uint4 *>(h->d_crec);
             s.smem_bytes = (uint32_t)h->host.split.size();
             s.s_dense = h->host.s_dense;
             s.s_rec = h->host.s_rec;
@@ -254,8 +259,6 @@ static void free_device(ac_stt *h) {
     h->d_stt2 = nullptr;
     cudaFree(h->d_split);
     h->d_split = nullptr;
-    cudaFree(h->d_crec);
-    h->d_crec = nullptr;
     cudaFree(h->d_class_map);
     cudaFree(h->d_out_off);
     cudaFree(h->d_out_ids);
@@ -286,8 +289,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         return AC_ERR_TOO_LARGE;
     }
     uint32_t kernel = opts ? opts->kernel : AC_KERNEL_AUTO;
-    if (opts && (opts->text_policy > 2 || opts->stt_policy > 2)) {
-        set_error("text_policy and stt_policy must be 0, 1 or 2");
+    if (opts && (opts->text_policy > 3 || opts->text_promotion > 4)) {
+        set_error("text_policy must be 0..3 and text_promotion 0..4");
         return AC_ERR_INVALID_ARG;
     }
     if (kernel > AC_KERNEL_GLOBAL) {
@@ -325,14 +328,13 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     if (variant == 0) {
         variant = kAutoVariant;
         if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
-        if (h->tier == AC_TIER_SPLIT && h->host.split.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
+        if (h->tier == AC_TIER_SPLIT) variant = kLeanVariant;
     }
     if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, variant)) {
         set_error("staged variant " + std::to_string(variant) + " has no room for the COMPACT table");
         return AC_ERR_INVALID_ARG;
     }
     SttView sg = view_of(h, 0), ss = view_of(h, variant);
-    ss.stt_evict_last = opts && opts->stt_policy == 2 ? 1u : 0u;
     // the two-byte walk exists for the two 32-warp x 16-byte shapes only
     if ((opts && opts->stride == 1) || (variant != 4 && variant != 7)) ss.stt2 = nullptr;
     const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
@@ -370,7 +372,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             g.n_readable = n_total - head;
             const uint32_t tp = opts ? opts->text_policy : 0;
             g.text_evict_first =
-                tp ? (tp == 2 ? 1u : 0u)
+                tp ? tp - 1u
                    : (tier_s == AC_TIER_GLOBAL || tier_s == AC_TIER_HYBRID || tier_s == AC_TIER_SPLIT) ? 1u : 0u;
             PFN_cuTensorMapEncodeTiled_v12000 enc = encode_fn();
             if (!enc) {
@@ -386,9 +388,13 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
                                            : W == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
                                            : W == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
                                                      : CU_TENSOR_MAP_SWIZZLE_NONE;
+            const uint32_t pr = opts ? opts->text_promotion : 0;
+            const CUtensorMapL2promotion promo = pr == 1   ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+                                                 : pr == 2 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+                                                 : pr == 3 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+                                                           : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
             CUresult cr = enc(&tmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, (void *)(d_text + head), dims, strides, box,
-                              estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                              estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz, promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
             if (cr != CUDA_SUCCESS) {
                 set_error("cuTensorMapEncodeTiled failed with CUresult " + std::to_string((int)cr));
                 return AC_ERR_CUDA;
@@ -820,7 +826,7 @@ ac_status ac_compile(const uint8_t *const *patterns, const uint32_t *lens, uint3
             o4.entry_bytes = 4;
         }
         rc = compile_table(patterns, lens, n, split ? &o4 : opts, *t);
-        if (rc == AC_OK && split && !split_table(*t, kDefaultCompactBudget)) {
+        if (rc == AC_OK && split && !split_table(*t, kDefaultSplitBudget)) {
             set_error("the automaton has no SPLIT encoding for the default shared-memory budget");
             rc = AC_ERR_TOO_LARGE;
         }
@@ -871,14 +877,11 @@ static void fill_info(const ac_table &t, ac_stt_info *info) {
     info->split_dstride = t.s_dstride;
     info->split_cold_records = t.s_cold_rec;
     info->split_bytes = t.split.size();
-    info->split_cold_full = t.s_cold_full;
-    info->split_crec_bytes = (uint64_t)t.crec.size() * 4;
 }
 
-ac_status ac_table_export_split(const ac_table *t, void *blob, uint32_t *crec) {
+ac_status ac_table_export_split(const ac_table *t, void *blob) {
     if (!t || t->split.empty() || !blob) return AC_ERR_INVALID_ARG;
     std::memcpy(blob, t->split.data(), t->split.size());
-    if (crec) std::memcpy(crec, t->crec.data(), t->crec.size() * 4);
     return AC_OK;
 }
 
@@ -994,7 +997,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             }
             h->host = std::move(t4);
         }
-        if (!split_table(h->host, cbudget)) {
+        if (!split_table(h->host, stt_budget(h, kSplitVariant))) {
             delete h;
             set_error("the automaton has no SPLIT encoding for the shared-memory budget");
             return AC_ERR_TOO_LARGE;
@@ -1058,9 +1061,6 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             return fail(e, "cudaMalloc(split)");
         if ((e = cudaMemcpy(h->d_split, t.split.data(), t.split.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
             return fail(e, "H2D split");
-        if ((e = cudaMalloc(&h->d_crec, t.crec.size() * 4)) != cudaSuccess) return fail(e, "cudaMalloc(crec)");
-        if ((e = cudaMemcpy(h->d_crec, t.crec.data(), t.crec.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess)
-            return fail(e, "H2D crec");
     }
     const std::vector<uint8_t> &blob = tier == AC_TIER_COMPACT ? t.compact : t.stt;
     const size_t stt_alloc = (blob.size() + 15) / 16 * 16 + 16;

@@ -39,9 +39,8 @@ struct ac_table {
     // SPLIT tier (ac_split.cpp): dense rows for BFS ids [0, s_dense) (s_dstride
     // u16 entries each), then s_rec 8-byte records for ids [s_dense, s_dense +
     // s_rec); every other state is read from the global 32-bit table
-    uint32_t s_dense = 0, s_rec = 0, s_dstride = 0, s_cold_rec = 0, s_cold_full = 0;
+    uint32_t s_dense = 0, s_rec = 0, s_dstride = 0, s_cold_rec = 0;
     std::vector<uint8_t> split;
-    std::vector<uint32_t> crec;  // SPLIT cold records, 4 words per state (global memory)
 
     // two-byte table (NEXT-4), built by stride2_table(): row s, column
     // c1 * n_classes + c2 -> delta(delta(s,c1),c2) | final flag << 31 |
@@ -59,7 +58,6 @@ struct ac_stt {
     void *d_stt = nullptr;           // entries
     uint32_t *d_stt2 = nullptr;      // two-byte table (NEXT-4) or NULL
     void *d_split = nullptr;         // SPLIT tier: the shared-memory part (dense rows + records)
-    uint32_t *d_crec = nullptr;      // SPLIT tier: 16-byte cold records of every state
     uint8_t *d_class_map = nullptr;  // 256 B
     uint32_t *d_out_off = nullptr;
     uint32_t *d_out_ids = nullptr;

@@ -142,38 +142,6 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
     return sp ? (need ? e3 : ex) : lo;
 }
 
-// SPLIT tier, cold lanes: the state's 16-byte cold record (global, L2
-// resident) -- three exceptions with 32-bit targets over the shared-memory
-// row of fd -- and, for states with more exceptions or an escaped row entry,
-// the full dense table.  The record loads carry an L2 evict-last hint when
-// st.stt_evict_last is set (the instruction-level form of an L2
-// access-policy window over the cold part of the automaton).
-__device__ __forceinline__ uint32_t split_cold(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
-    uint4 r;
-    if (st.stt_evict_last) {
-        uint64_t pol;
-        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-        asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
-                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
-                     : "l"(st.crec + s), "l"(pol));
-    } else {
-        r = __ldg(st.crec + s);
-    }
-    uint32_t row = s;  // full-table row to read if the record cannot answer
-    const uint32_t fd = r.x & 0xFFFFu;
-    if (fd != 0xFFFFu) {
-        const uint32_t x = r.x ^ (cls * 0x01010000u);
-        if ((x & 0x00FF0000u) == 0) return r.y;
-        if (x < 0x01000000u) return r.z;
-        if ((r.w & 0xFFu) == cls) return ((r.w >> 8) & 0x7FFFFFu) | (r.w & 0x80000000u);
-        uint32_t e = base + fd * st.s_row_bytes + cls * 2u;
-        asm("ld.shared.u16 %0, [%0];" : "+r"(e));
-        if (e != 0xFFFFu) return (e >> 1) | (e << 31);
-        row = fd;  // delta(s, cls) = delta(fd, cls), whose 16-bit entry escaped
-    }
-    return __ldg(static_cast<const uint32_t *>(st.stt) + ((size_t)row * st.stride + cls));
-}
-
 // SPLIT tier (ac_split.cpp): delta(s, cls) as a 32-bit entry (BFS id | flag
 // << 31) by one rule for every hot state: delta = t1 if cls == c1, t2 if
 // cls == c2, else row[fd][cls].  Only sparse hot states (s_dense <= s <
@@ -199,7 +167,15 @@ __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st,
         : "r"(h1 | h2));
     const uint32_t e16 = h1 ? (hi & 0xFFFFu) : h2 ? (hi >> 16) : e;
     uint32_t g = (e16 >> 1) | (e16 << 31);  // 2 x + flag -> x | flag << 31
-    if (e16 == 0xFFFFu) g = split_cold(base, st, s, cls);
+    if (e16 == 0xFFFFu) {
+        // cold: the full entry from the dense table through L1/L2.  (Measured
+        // slower: a 16-byte L2-resident cold record per state answering three
+        // exceptions over the shared-memory rows first -- the extra dependent
+        // load doubled the long-scoreboard stalls, C3 list 3.2 -> 5.4 ms/GiB;
+        // an L2 evict-last hint on this load: no change.)
+        const uint32_t *gp = static_cast<const uint32_t *>(st.stt) + ((size_t)s * st.stride + cls);
+        asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(g) : "l"(gp));
+    }
     return g;
 }
 
@@ -396,21 +372,6 @@ __device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t
     } else {
         cnt += c;
     }
-}
-
-// emit_outputs out of line, for tiers whose matches are rare (SPLIT): the
-// 16-byte walk loop is unrolled, and inlining the emission at every byte
-// multiplies its code past the instruction cache.  State goes in and out by
-// value so nothing is spilled to the stack.
-struct CntWp {
-    uint32_t cnt;
-    uint64_t wp;
-};
-template <typename E, int TIER, int MODE>
-__device__ __noinline__ CntWp emit_outputs_rare(uint32_t x, uint64_t key0, uint32_t cnt, uint64_t wp, const E *s_stt,
-                                                const SttView &st, const ScanOut &so) {
-    emit_outputs<E, TIER, MODE>(x, key0, cnt, wp, s_stt, st, so);
-    return CntWp{cnt, wp};
 }
 
 // One transition inside the owned chunk: count or emit output(s) at the
@@ -857,7 +818,12 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
     const bool tma_halo = (uint64_t)nh0 * W <= L;  // the halo window lies inside the next chain
     const uint32_t nh = tma_halo ? nh0 : 0;
     const uint32_t m = idle ? 0u : nh + (uint32_t)(L / W);
-    const uint64_t pol = text_l2_policy(g.text_evict_first);
+    // text_evict_first: 0 = evict-normal, 1 = evict-first, 2 = per 32-byte
+    // sector: the half a chain reads first (the upper one, the walk is right
+    // to left) evict-normal, the second half evict-first -- a 16-byte box
+    // pulls a whole sector, so the first half keeps it for the second
+    const uint64_t pol = text_l2_policy(g.text_evict_first != 0);
+    const uint64_t pol_first_half = g.text_evict_first == 2 ? text_l2_policy(0) : pol;
 
     auto issue = [&](uint32_t j) {
         const uint32_t slot = j % NST;
@@ -870,7 +836,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
             y = (int)row0;
         }
         mbar_expect_tx(&wbar[slot], Sh::SLOT);
-        tma_load_2d(wring + slot * Sh::SLOT, &tmap, x, y, &wbar[slot], pol);
+        tma_load_2d(wring + slot * Sh::SLOT, &tmap, x, y, &wbar[slot], (x & 16) ? pol_first_half : pol);
     };
     if (lane == 0)
         for (uint32_t j = 0; j < (uint32_t)NST && j < m; j++) issue(j);
@@ -925,6 +891,39 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
             }
         } else {
             const uint64_t col0 = L - (uint64_t)(j - nh + 1) * W;
+            // single-slot ring (NST = 1): the lane copies its whole W-byte
+            // row into registers and the slot is refilled at once, so the
+            // next box's TMA overlaps the walk of this one; with 32-byte
+            // boxes every 32-byte sector of the text is fetched exactly once
+            // (a 16-byte box pulls a whole sector, and with the text's
+            // evict-first policy the second half was often re-fetched)
+            uint4 vall[NST == 1 ? W / 16 : 1][K];
+            if constexpr (NST == 1) {
+#pragma unroll
+                for (int q = 0; q < W / 16; q++)
+#pragma unroll
+                    for (int k = 0; k < K; k++) {
+                        const uint32_t logical = (k * 32 + lane) * W + q * 16;
+                        vall[q][k] =
+                            *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
+                    }
+                // the slot may be overwritten only once every lane's loads have
+                // landed: an opaque zero computed from the loaded words,
+                // OR-reduced over the warp (the scoreboard waits for every
+                // lane's loads), feeds the next box index; then the
+                // generic-to-async proxy fence before the TMA write
+                uint32_t dep = 0;
+#pragma unroll
+                for (int q = 0; q < W / 16; q++)
+#pragma unroll
+                    for (int k = 0; k < K; k++) dep |= vall[q][k].x | vall[q][k].y | vall[q][k].z | vall[q][k].w;
+                dep &= (uint32_t)(g.n_chains >> 63);  // 0, but not a compile-time constant
+                dep = __reduce_or_sync(0xffffffffu, dep);
+                if (lane == 0 && j + 1 < m) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    issue(j + 1 + dep);
+                }
+            }
 #pragma unroll
             for (int q = W / 16 - 1; q >= 0; --q) {
                 uint4 v[K];
@@ -932,7 +931,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
                 for (int k = 0; k < K; k++) {
                     const uint32_t logical = (k * 32 + lane) * W + q * 16;
-                    v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
+                    if constexpr (NST == 1)
+                        v[k] = vall[q][k];
+                    else
+                        v[k] = *reinterpret_cast<const uint4 *>(tile + (logical ^ (((logical >> 7) & Sh::SWZ) << 4)));
                     kb[k] = (so.base + g.m0 + cbase[k] + col0 + q * 16) << 24;
                 }
                 // (COMPACT counting keeps its predicated per-byte count: measured faster)
@@ -1075,16 +1077,11 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                             const uint32_t e =
                                 next_entry<E, TIER>(s_stt, st, s[k], class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
                             s[k] = state_of<E, TIER>(e, st);
-                            if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k]) {
-                                if constexpr (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT) {
-                                    const CntWp r = emit_outputs_rare<E, TIER, MODE>(
-                                        s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt, st, so);
-                                    cnt[k] = r.cnt;
-                                    wp[k] = r.wp;
-                                } else {
-                                    cnt[k] += out_count<E, TIER>(s_stt, st, s[k]);
-                                }
-                            }
+                            // (an out-of-line emission call was measured slower: C3 list
+                            // 1.05 -> 1.30 ms per 256 MiB)
+                            if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k])
+                                emit_outputs<E, TIER, MODE>(s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
+                                                            st, so);
                         }
                     }
                 } else {
@@ -1098,8 +1095,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                 }
             }
         }
-        __syncwarp();  // every lane is done with this slot
-        if (lane == 0 && j + NST < m) issue(j + NST);
+        if (NST > 1 || j < nh) {  // (NST = 1 main boxes refilled their slot above)
+            __syncwarp();              // every lane is done with this slot
+            if (lane == 0 && j + NST < m) issue(j + NST);
+        }
     }
 
     if constexpr (MODE == MODE_COUNT_CHAINS || MODE == MODE_EMIT_OPT) {

@@ -46,10 +46,8 @@ struct SttView {
     // s_rec_x0 + 8 s (biased by -8 s_dense, wraps);
     // `stt` stays the full 32-bit table for the cold states
     const void *sblob;
-    const uint4 *crec;  // cold records (global, 16 B per state)
     uint32_t s_dense, s_rec, s_row_bytes, s_rec_x0;
     uint32_t cmap_ident;  // the class map is the identity (every byte occurs in a pattern)
-    uint32_t stt_evict_last;  // SPLIT: cold global-table loads carry an L2 evict-last hint
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.
@@ -115,7 +113,7 @@ struct StagedGeom {
     uint64_t n_chains;     // full chains in the main region
     uint64_t chain0;       // global index of main chain 0
     uint64_t n_readable;   // bytes readable from the main-region pointer (halo bound)
-    uint32_t text_evict_first;  // L2 policy of the text's TMA loads (see text_l2_policy)
+    uint32_t text_evict_first;  // L2 policy of the text's TMA loads: 0 normal, 1 evict-first, 2 per-sector pair
 };
 
 struct StagedConfig {
@@ -136,7 +134,8 @@ struct StagedConfig {
     X(6, 32, 2, 16, 2, 1)     \
     X(7, 32, 1, 16, 2, 1)     \
     X(8, 32, 1, 32, 2, 0)     \
-    X(9, 16, 2, 16, 2, 1)
+    X(9, 16, 2, 16, 2, 1)     \
+    X(10, 32, 1, 32, 1, 1)
 
 // Kernel entry points (host side launchers); all return cudaError_t.
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,

@@ -30,19 +30,10 @@
 //   * states >= H are COLD: the kernel does not read a record for them.
 // A 16-bit entry is 2 x + flag (x = BFS id of the next state, flag =
 // output(x) != {}) when x < 32767, else 0xFFFF; 0xFFFF (cold state, cold
-// record, large id) sends the lane to global memory:
-//   * first the COLD RECORD of s, 16 bytes per state (2 MB for C3, so it
-//     stays L2-resident next to the streamed text):
-//       w0 = fd | c1 << 16 | c2 << 24, w1 = t1, w2 = t2, w3 = c3 | t3 << 8
-//     the same rule with three exceptions and 32-bit (24-bit for t3)
-//     entries, fd = the first dense state on s's failure chain (whose row is
-//     in shared memory);
-//   * states needing more exceptions (fd = 0xFFFF), and dense-row entries
-//     that escaped, read the full 32-bit dense table (the paper's STT,
-//     P:118) -- 137 MB for C3, mostly DRAM-resident, now touched by < 1 % of
-//     the steps.
-// Output enumeration always reads that table's per-row output summary
-// (matches are rare where this tier is chosen).
+// record, large id) sends the lane to the full 32-bit dense table in global
+// memory (L1/L2; the paper's STT).  Output enumeration always reads
+// that table's per-row output summary (matches are rare where this tier is
+// chosen).
 #include <algorithm>
 #include <cstring>
 
@@ -132,30 +123,7 @@ bool split_table(ac_table &t, size_t budget) {
         std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8], &lo, 4);
         std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8 + 4], &hi, 4);
     }
-    // cold records of every state (dense states: marker, never used)
-    std::vector<uint32_t> crec((size_t)S * 4, 0);
-    uint32_t n_cold_full = 0;
-    for (uint32_t s = 0; s < S; s++) {
-        uint32_t *r = &crec[(size_t)s * 4];
-        uint32_t cls[3] = {0, 0, 0};
-        const uint32_t k = s < D ? 4u : exceptions(s, fd[s], cls, 3);
-        if (k == 0) cls[0] = 0;
-        if (k <= 1) cls[1] = cls[0];
-        if (k <= 2) cls[2] = cls[1];
-        const uint32_t t3 = delta(s, cls[2]);
-        if (k > 3 || (t3 & 0x7fffffffu) >= (1u << 23)) {
-            r[0] = 0xFFFFu;  // read the dense global row
-            n_cold_full += s >= D;
-            continue;
-        }
-        r[0] = fd[s] | (cls[0] << 16) | (cls[1] << 24);
-        r[1] = delta(s, cls[0]);
-        r[2] = delta(s, cls[1]);
-        r[3] = cls[2] | ((t3 & 0x7fffffu) << 8) | ((t3 >> 31) << 31);
-    }
     t.split.swap(blob);
-    t.crec.swap(crec);
-    t.s_cold_full = n_cold_full;
     t.s_dense = D;
     t.s_rec = H;
     t.s_dstride = dstride;

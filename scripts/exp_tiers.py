@@ -39,6 +39,7 @@ def main():
     p.add_argument("--tiers", default="global,split")
     p.add_argument("--variants", default="0")
     p.add_argument("--list", action="store_true")
+    p.add_argument("--exact-cap", action="store_true", help="list buffer of exactly count records")
     p.add_argument("--policies", default="0", help="text L2 policies (0 auto, 1 evict-normal, 2 evict-first)")
     a = p.parse_args()
     for name in a.workloads.split(","):
@@ -52,10 +53,11 @@ def main():
             except ac.AcError as e:
                 print(json.dumps({"workload": name, "tier": tname, "skipped": str(e)}), flush=True)
                 continue
-            out = torch.empty(n // 8 + 64, dtype=torch.int64, device="cuda") if a.list else None
+            cap = ac.count(stt, text) if a.exact_cap else n // 8 + 64
+            out = torch.empty(max(1, cap), dtype=torch.int64, device="cuda") if a.list else None
             for v, pol in [(v, pol) for v in a.variants.split(",") for pol in a.policies.split(",")]:
-                tpol, spol = (pol + ":0").split(":")[:2]  # text policy[:stt policy]
-                knobs = dict(kernel=ac.KERNEL_STAGED, variant=int(v), text_policy=int(tpol), stt_policy=int(spol))
+                tpol, prom = (pol + ":0").split(":")[:2]  # text policy[:promotion]
+                knobs = dict(kernel=ac.KERNEL_STAGED, variant=int(v), text_policy=int(tpol), text_promotion=int(prom))
                 try:
                     ac.match_async(stt, text, out, res, **knobs)
                 except ac.AcError as e:
@@ -63,7 +65,7 @@ def main():
                     continue
                 t = timeit(lambda: ac.match_async(stt, text, out, res, **knobs))
                 print(json.dumps({"workload": name, "n": n, "tier": stt.tier_name, "variant": int(v),
-                                  "policy": pol, "list": bool(a.list),
+                                  "policy": pol, "list": bool(a.list), "exact_cap": bool(a.exact_cap),
                                   "states": stt.info["n_states"], "split_dense": stt.info["split_dense"],
                                   "split_records": stt.info["split_records"], "ms": round(t, 4),
                                   "gbps": round(n * 8 / t / 1e6, 1), "matches": int(res[0]),
