@@ -45,6 +45,13 @@
 
 namespace acx {
 
+#ifdef AC_DEBUG_TIMES
+// debug builds (AC_EXTRA_NVCC_FLAGS=-DAC_DEBUG_TIMES): per-warp walk times of
+// the staged scan (one copy per translation unit; ac_tier_split.cu exports
+// ac_debug_times() for its own)
+static __device__ unsigned long long ac_dbg_times[1024 * 32 * 2];
+#endif
+
 static constexpr int GT = 256;  // k_scan_global block size
 
 template <typename E>
@@ -805,6 +812,10 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
         if (so.res->status != AC_OK) return;  // capacity exceeded: write nothing
     }
     const uint32_t tile = s_tile;
+#ifdef AC_DEBUG_TIMES
+    uint64_t dbg_t0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(dbg_t0));
+#endif
     const uint64_t row0 = (uint64_t)tile * (WARPS * Sh::ROWS) + (uint64_t)warp * Sh::ROWS;
     // in-kernel placement ends with CTA barriers: idle warps stay (no tiles)
     const bool idle = row0 >= g.n_chains;
@@ -1101,6 +1112,16 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
         }
     }
 
+#ifdef AC_DEBUG_TIMES
+    if (lane == 0 && tile < 1024 && warp < 32) {  // debug build only: walk time of each warp
+        uint64_t t1;
+        uint32_t smid;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        ac_dbg_times[(tile * 32 + warp) * 2] = dbg_t0;
+        ac_dbg_times[(tile * 32 + warp) * 2 + 1] = (t1 - dbg_t0) | ((uint64_t)smid << 48);
+    }
+#endif
     if constexpr (MODE == MODE_COUNT_CHAINS || MODE == MODE_EMIT_OPT) {
 #pragma unroll
         for (int k = 0; k < K; k++)

@@ -9,3 +9,9 @@ template cudaError_t launch_staged_tier<AC_TIER_SPLIT>(int, uint32_t, int, const
                                                     const SttView &, const StagedGeom &, const ScanOut &, size_t,
                                                     cudaStream_t);
 }  // namespace acx
+
+#ifdef AC_DEBUG_TIMES
+extern "C" int ac_debug_times(unsigned long long *host, unsigned n) {
+    return (int)cudaMemcpyFromSymbol(host, acx::ac_dbg_times, n * sizeof(unsigned long long));
+}
+#endif
