@@ -974,18 +974,22 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     // prefix reached through generic loads, so AUTO never picks HYBRID
     const size_t cbudget = stt_budget(h, kLeanVariant);
     const uint32_t want_stride = opts ? opts->stride : 0;
+    bool auto_split = false;
     if (tier == AC_TIER_AUTO) {
         if (stt_bytes <= budget) tier = AC_TIER_SMEM;
         else if (compact_table(h->host, cbudget)) tier = AC_TIER_COMPACT;
         // small alphabets (DNA): the L1/L2 table with two bytes per lookup
         else if (t.n_classes <= 8 && want_stride != 1 && t.entry_bytes == 4) tier = AC_TIER_GLOBAL;
-        else tier = AC_TIER_SPLIT;
+        else tier = AC_TIER_SPLIT, auto_split = true;
     }
     if (tier == AC_TIER_SPLIT) {
-        if (t.entry_bytes != 4) {  // the cold states need the 32-bit global table: rebuild it so
+        // the cold states need the 32-bit global table: build it if the
+        // dictionary compiled to 16-bit entries
+        ac_table t4;
+        ac_table *ts = &h->host;
+        if (t.entry_bytes != 4) {
             ac_build_opts o = opts ? *opts : ac_build_opts{sizeof(ac_build_opts), 0, 0, 0, 0, 0};
             o.entry_bytes = 4;
-            ac_table t4;
             try {
                 rc = compile_table(patterns, lens, n, &o, t4);
             } catch (...) {
@@ -995,14 +999,25 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
                 delete h;
                 return rc;
             }
-            h->host = std::move(t4);
+            ts = &t4;
         }
-        if (!split_table(h->host, stt_budget(h, kSplitVariant))) {
+        const bool ok = split_table(*ts, stt_budget(h, kSplitVariant));
+        // AUTO keeps SPLIT only where its shared-memory part covers the hot
+        // automaton: measured, it loses to the plain L1/L2 table when many
+        // sparse hot states need more than two exceptions (C5 Snort 50K
+        // patterns, 47 % cold records: 3.95 vs 1.98 ms; English 5K, 26 %:
+        // 6.2 vs 2.5 ms; C3, 6.5 %: 0.60 vs 0.80 ms count)
+        const bool good = ok && 20u * ts->s_cold_rec <= 3u * (ts->s_rec - ts->s_dense);
+        if (auto_split && !good) {
+            tier = AC_TIER_GLOBAL;
+        } else if (!ok) {
             delete h;
             set_error("the automaton has no SPLIT encoding for the shared-memory budget");
             return AC_ERR_TOO_LARGE;
+        } else {
+            if (ts != &h->host) h->host = std::move(t4);
+            hot = h->host.s_rec;
         }
-        hot = h->host.s_dense + h->host.s_rec;
     }
     if (tier == AC_TIER_COMPACT) {
         if (h->host.compact.empty() && !compact_table(h->host, cbudget)) {

@@ -1076,11 +1076,39 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                                                     kb[k] + ((uint64_t)bb << 24), kb[k] + ((uint64_t)(bb - 1) << 24),
                                                     live[k], s_cmap, s_stt, st, so);
                     }
-                } else if constexpr (TIER == AC_TIER_SPLIT) {
+                } else if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT)) {
                     // rare matches (the tier is chosen for large byte
-                    // dictionaries): the walk is the whole loop body; the
-                    // record key and the chain's liveness are only touched
-                    // on a flagged byte
+                    // dictionaries): the 16 steps only collect the flag bits
+                    // -- the count-mode loop, no record keys or slot
+                    // pointers live in it -- and a lane that saw a flag
+                    // re-walks the chunk from its first state, emitting
+                    // (C3: 0.5 % of lane-chunks, 15 % of warp-chunks)
+#pragma unroll
+                    for (int k = 0; k < K; k++) {
+                        const uint32_t s_in = s[k];
+                        uint32_t fm = 0;
+#pragma unroll
+                        for (int bb = 15; bb >= 0; --bb) {
+                            const uint32_t e =
+                                next_entry<E, TIER>(s_stt, st, s[k], class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                            s[k] = state_of<E, TIER>(e, st);
+                            fm |= flag_of<E, TIER>(e, s[k], st) << bb;
+                        }
+                        if (__any_sync(0xffffffffu, fm != 0 && live[k]) && fm != 0 && live[k]) {
+                            uint32_t x = s_in;
+#pragma unroll 1
+                            for (int bb = 15; bb >= 0; --bb) {
+                                const uint32_t e = next_entry<E, TIER>(
+                                    s_stt, st, x, class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                                x = state_of<E, TIER>(e, st);
+                                if ((fm >> bb) & 1u)
+                                    emit_outputs<E, TIER, MODE>(x, kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
+                                                                st, so);
+                            }
+                        }
+                    }
+                } else if constexpr (TIER == AC_TIER_SPLIT) {
+                    // counting with rare matches: the walk is the whole loop
 #pragma unroll
                     for (int bb = 15; bb >= 0; --bb) {
 #pragma unroll
@@ -1088,8 +1116,6 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                             const uint32_t e =
                                 next_entry<E, TIER>(s_stt, st, s[k], class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
                             s[k] = state_of<E, TIER>(e, st);
-                            // (an out-of-line emission call was measured slower: C3 list
-                            // 1.05 -> 1.30 ms per 256 MiB)
                             if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k])
                                 emit_outputs<E, TIER, MODE>(s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
                                                             st, so);
