@@ -1002,12 +1002,15 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             ts = &t4;
         }
         const bool ok = split_table(*ts, stt_budget(h, kSplitVariant));
-        // AUTO keeps SPLIT only where its shared-memory part covers the hot
-        // automaton: measured, it loses to the plain L1/L2 table when many
-        // sparse hot states need more than two exceptions (C5 Snort 50K
-        // patterns, 47 % cold records: 3.95 vs 1.98 ms; English 5K, 26 %:
-        // 6.2 vs 2.5 ms; C3, 6.5 %: 0.60 vs 0.80 ms count)
-        const bool good = ok && 20u * ts->s_cold_rec <= 3u * (ts->s_rec - ts->s_dense);
+        // AUTO keeps SPLIT where the plain table would live in DRAM (> 32 MiB;
+        // a table that fits L2 beside the streamed text is served well by
+        // L1/L2: C5 Snort 1K, 15 MB: 0.43 ms GLOBAL vs 0.55 SPLIT per 256
+        // MiB list) and the shared-memory part covers the hot automaton
+        // (<= 30 % of the sparse hot states are cold records: Snort 50K, 46 %:
+        // 1.12 GLOBAL vs 1.63 SPLIT; Snort 20K, 22 %: 1.00 vs 0.80; Snort 5K,
+        // 4 %: 0.68 vs 0.59; C3, 7 %: 0.80 vs 0.66)
+        const bool big = (uint64_t)ts->n_states * ts->row_stride * 4 > (32ull << 20);
+        const bool good = ok && big && 10u * ts->s_cold_rec <= 3u * (ts->s_rec - ts->s_dense);
         if (auto_split && !good) {
             tier = AC_TIER_GLOBAL;
         } else if (!ok) {

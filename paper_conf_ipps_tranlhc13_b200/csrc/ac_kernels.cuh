@@ -180,7 +180,8 @@ __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st,
         // exceptions over the shared-memory rows first -- the extra dependent
         // load doubled the long-scoreboard stalls, C3 list 3.2 -> 5.4 ms/GiB;
         // an L2 evict-last hint on this load: no change.)
-        const uint32_t *gp = static_cast<const uint32_t *>(st.stt) + ((size_t)s * st.stride + cls);
+        // (S x row_stride < 2^32 entries, checked by ac_build: a 32-bit index)
+        const uint32_t *gp = static_cast<const uint32_t *>(st.stt) + (s * st.stride + cls);
         asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(g) : "l"(gp));
     }
     return g;
