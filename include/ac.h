@@ -208,6 +208,12 @@ typedef struct {
     uint32_t text_promotion; /* L2 promotion of the text's TMA misses:
                               0 = auto (256 B), 1 = none, 2 = 64 B,
                               3 = 128 B, 4 = 256 B (ablation knob)          */
+    uint32_t l2_window_mib; /* > 0: the staged scan runs with a persisting L2
+                              access-policy window over the first MiB of the
+                              global table (GLOBAL/HYBRID/SPLIT tiers; capped
+                              by the device's persisting-L2 limit, which the
+                              first such call raises to its maximum -- a
+                              process-wide setting).  0 = off (default)      */
 } ac_match_opts;
 
 /* Per-call device result written by the async entry points. */

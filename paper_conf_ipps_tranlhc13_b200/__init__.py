@@ -75,7 +75,8 @@ class ac_match_opts(ctypes.Structure):
                 ("stride", ctypes.c_uint32),
                 ("n_events", ctypes.c_uint32),
                 ("events", ctypes.POINTER(ctypes.c_void_p)),
-                ("text_policy", ctypes.c_uint32), ("text_promotion", ctypes.c_uint32)]
+                ("text_policy", ctypes.c_uint32), ("text_promotion", ctypes.c_uint32),
+                ("l2_window_mib", ctypes.c_uint32)]
 
 
 _lib = None
@@ -209,9 +210,10 @@ def _check_text(text: torch.Tensor):
 
 
 def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, scratch_slots: int = 0,
-           two_pass: bool = False, events=None, stride: int = 0, text_policy: int = 0, text_promotion: int = 0):
+           two_pass: bool = False, events=None, stride: int = 0, text_policy: int = 0, text_promotion: int = 0,
+           l2_window_mib: int = 0):
     o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, scratch_slots,
-                      int(two_pass), stride, 0, None, text_policy, text_promotion)
+                      int(two_pass), stride, 0, None, text_policy, text_promotion, l2_window_mib)
     if events:
         arr = (ctypes.c_void_p * (2 * len(events)))(*[e.cuda_event for pair in events for e in pair])
         o.n_events = len(events)
@@ -223,7 +225,7 @@ def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, sc
 def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: torch.Tensor, *,
                 n_halo: int = 0, base: int = 0, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0,
                 variant: int = 0, scratch_slots: int = 0, two_pass: bool = False, stride: int = 0,
-                events=None, text_policy: int = 0, text_promotion: int = 0) -> int:
+                events=None, text_policy: int = 0, text_promotion: int = 0, l2_window_mib: int = 0) -> int:
     """Enqueue the scan; result (int64[2] CUDA) receives (count, status).
     ``text`` holds n_owned + n_halo bytes.  ``kernel``/``chain_bytes``/
     ``variant``/``scratch_slots``/``two_pass`` select the scan (ac_match_opts).  ``events``: optional list
@@ -244,7 +246,8 @@ def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: 
         cap = out.numel()
         # non-NULL selects list mode; with cap == 0 the status gates every write
         optr = out.data_ptr() if cap else result.data_ptr()
-    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events, stride, text_policy, text_promotion)
+    o = _mopts(kernel, chain_bytes, variant, scratch_slots, two_pass, events, stride, text_policy, text_promotion,
+               l2_window_mib)
     L = lib()
     _check(L.ac_match_async(stt.handle, text.data_ptr() if n_total else None, n_total - n_halo, n_halo, base,
                             optr, cap, result.data_ptr(), _stream_ptr(stream), ctypes.byref(o)))

@@ -338,6 +338,22 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     // the two-byte walk exists for the two 32-warp x 16-byte shapes only
     if ((opts && opts->stride == 1) || (variant != 4 && variant != 7)) ss.stt2 = nullptr;
     const uint32_t tier_g = tier_of(h, sg), tier_s = tier_of(h, ss);
+    // l2_window_mib > 0: persisting L2 window over that many MiB of the
+    // global table (tiers that read it: GLOBAL, HYBRID, SPLIT), capped by the
+    // device's persisting L2 limit, which the first such call raises
+    size_t win_bytes = 0;
+    if (opts && opts->l2_window_mib && tier_s != AC_TIER_SMEM && tier_s != AC_TIER_COMPACT) {
+        size_t lim = 0;
+        if (cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize) == cudaSuccess && lim == 0) {
+            cudaDeviceProp pr;
+            if (cudaGetDeviceProperties(&pr, h->device) == cudaSuccess)
+                cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)pr.persistingL2CacheMaxSize);
+            cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize);
+        }
+        cudaGetLastError();
+        const size_t tbl = (size_t)h->host.n_states * row_bytes(h);
+        win_bytes = std::min<size_t>({(size_t)opts->l2_window_mib << 20, tbl, lim});
+    }
     const size_t smem_g = smem_of(h, sg), smem_s = smem_of(h, ss);
     const StagedConfig cfg = staged_variant(variant);
 
@@ -448,8 +464,27 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             pre(stream);
             ScanOut sso = so;
             if (mode == MODE_EMIT_OPT) sso.nbits = nm_bits;
-            AC_CUDA(launch_scan_staged(mode, eb, tier_s, variant, tmap, d_text + g.m0, ss, g, sso, smem_s, stream),
-                    sname);
+            // optional L2 access-policy window (SURVEY 8(a)-a5 tier (iii)) over
+            // the hottest rows of the global table (BFS order: shallow rows
+            // first), set on the stream for this launch only
+            const bool apw = win_bytes > 0;
+            if (apw) {
+                cudaStreamAttrValue v = {};
+                v.accessPolicyWindow.base_ptr = h->d_stt;
+                v.accessPolicyWindow.num_bytes = win_bytes;
+                v.accessPolicyWindow.hitRatio = 1.0f;
+                v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+                v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+                AC_CUDA(cudaStreamSetAttribute(stream, cudaStreamAttributeAccessPolicyWindow, &v),
+                        "cudaStreamSetAttribute(access policy window)");
+            }
+            const cudaError_t le =
+                launch_scan_staged(mode, eb, tier_s, variant, tmap, d_text + g.m0, ss, g, sso, smem_s, stream);
+            if (apw) {
+                cudaStreamAttrValue v = {};  // num_bytes = 0: the caller's later launches are unaffected
+                cudaStreamSetAttribute(stream, cudaStreamAttributeAccessPolicyWindow, &v);
+            }
+            AC_CUDA(le, sname);
             post(sname, stream, g.n_chains * g.chain_len);
         }
         if (side) AC_CUDA(cudaStreamWaitEvent(stream, side->join, 0), "cudaStreamWaitEvent(join)");

@@ -150,31 +150,34 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
 }
 
 // SPLIT tier (ac_split.cpp): delta(s, cls) as a 32-bit entry (BFS id | flag
-// << 31) by one rule for every hot state: delta = t1 if cls == c1, t2 if
-// cls == c2, else row[fd][cls].  Only sparse hot states (s_dense <= s <
-// s_rec) load their 8-byte record; the others start from (fd = s for a
-// dense state, fd = the all-0xFFFF escape row for a cold one; exception
-// classes ~cls, which never match), so every lane runs the same
-// instructions.  A 16-bit result of 0xFFFF -- cold state, cold record or a
-// next id >= 32767 -- is replaced by the full entry from the global table
-// (L1/L2).
+// << 31).  A hot state of the record level (s_dense <= s < s_rec) loads its
+// children record {c1..c4 | fd, first, flags}: delta = first + k if cls ==
+// c_k, else row[fd][cls]; a dense state reads row[s][cls]; a cold state
+// (s >= s_rec) reads the escape row.  Every lane runs the same instructions
+// (the class bytes of a non-record lane are cls ^ 0x80, which never match).
+// A 16-bit result above 0xFFFD -- cold state, cold record or a next id >=
+// 32767 -- is replaced by the full entry from the global table (L1/L2).
 __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
+    const uint32_t rep = cls * 0x01010101u;
     const uint32_t sparse = (s - st.s_dense) < (st.s_rec - st.s_dense);
-    uint32_t lo = min(s, st.s_dense) | ((cls ^ 0xFFu) * 0x01010000u);
-    uint32_t hi = base + st.s_rec_x0 + s * 8u;  // record address (biased by -8 s_dense)
-    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%1];\n\t}"
+    uint32_t lo = base + st.s_rec_x0 + s * 8u;  // record address (biased by -8 s_dense)
+    uint32_t hi = min(s, st.s_dense);           // fd of a dense state (itself) or of a cold one (escape row)
+    asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%0];\n\t"
+        "@!p xor.b32 %0, %3, 0x80808080;\n\t}"
         : "+r"(lo), "+r"(hi)
-        : "r"(sparse));
-    // lo = fd | c1 << 16 | c2 << 24, hi = t1 | t2 << 16
-    const uint32_t x = lo ^ (cls * 0x01010000u);  // c1, c2 bytes become 0 where they match
-    const uint32_t h1 = (x & 0x00FF0000u) == 0, h2 = x < 0x01000000u;
-    uint32_t e = base + (lo & 0xFFFFu) * st.s_row_bytes + cls * 2u;  // row[fd][cls]
+        : "r"(sparse), "r"(rep));
+    // lo = c1 | c2 << 8 | c3 << 16 | c4 << 24, hi = fd | first << 12 | flags << 27
+    const uint32_t x = lo ^ rep;                                  // a zero byte where a class matches
+    const uint32_t z = (x - 0x01010101u) & ~x & 0x80808080u;      // lowest set bit: the first match
+    const uint32_t kk = (__ffs(z) - 1u) >> 3;                      // child index (garbage if no match)
+    uint32_t e = base + (hi & 0xFFFu) * st.s_row_bytes + cls * 2u;  // row[fd][cls]
     asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
         : "+r"(e)
-        : "r"(h1 | h2));
-    const uint32_t e16 = h1 ? (hi & 0xFFFFu) : h2 ? (hi >> 16) : e;
+        : "r"(z));
+    const uint32_t child = ((((hi >> 12) & 0x7FFFu) + kk) << 1) | ((hi >> (27u + kk)) & 1u);
+    const uint32_t e16 = z ? child : e;
     uint32_t g = (e16 >> 1) | (e16 << 31);  // 2 x + flag -> x | flag << 31
-    if (e16 == 0xFFFFu) {
+    if (e16 > 0xFFFDu) {
         // cold: the full entry from the dense table through L1/L2.  (Measured
         // slower: a 16-byte L2-resident cold record per state answering three
         // exceptions over the shared-memory rows first -- the extra dependent

@@ -12,26 +12,24 @@
 // on the C3 text: depth 1 = 60 %, depth 2 = 38 %, deeper 2 %), and in the AC
 // automaton delta(s,c) = g(s,c) if the trie has that edge, else
 // delta(f(s),c) (P:62 with the failure function of P:52).  So, in BFS order
-// (states sorted by depth, the ids of the global dense table), the HOT
-// states [0, H) are served from shared memory by one rule:
+// (states sorted by depth, the ids of the global dense table):
 //
-//   record(s) = fd(s) | c1 << 16 | c2 << 24,  t1 | t2 << 16
-//   delta(s, c) = t1 if c == c1, t2 if c == c2, else row[fd(s)][c]
-//
-// where row[] are dense 16-bit rows, also in shared memory:
-//   * the shallow levels [0, D) are DENSE: no record is stored; the kernel
-//     uses (fd = s, no exception class), i.e. reads the state's own row;
-//   * the next states [D, H) are SPARSE: fd(s) = the first dense state on s's
-//     failure chain, (c1, t1), (c2, t2) = the (at most two) classes where
-//     delta(s,.) differs from delta(fd(s),.) -- repeated, or (0, delta(s, 0)),
-//     when there are fewer, so every stored pair is exactly delta(s, c);
-//   * a sparse state needing more exceptions is COLD: its record points at
-//     row[D], the ESCAPE row (all 0xFFFF), with t1 = t2 = 0xFFFF;
-//   * states >= H are COLD: the kernel does not read a record for them.
-// A 16-bit entry is 2 x + flag (x = BFS id of the next state, flag =
-// output(x) != {}) when x < 32767, else 0xFFFF; 0xFFFF (cold state, cold
-// record, large id) sends the lane to the full 32-bit dense table in global
-// memory (L1/L2; the paper's STT).  Output enumeration always reads
+//   * the shallow levels [0, D) are DENSE: 16-bit rows in shared memory
+//     (the levels whose states mostly have more than four children);
+//   * the next level [D, H) gets an 8-byte CHILDREN record per state:
+//       lo = c1 | c2 << 8 | c3 << 16 | c4 << 24   (children's classes, ascending)
+//       hi = fd | first << 12 | flags << 27
+//     delta(s, c) = first + k if c == c_k (k = 0..3: BFS numbers a state's
+//     children consecutively in class order), else row[fd][c] -- fd = f(s),
+//     which is dense, so the exceptions of s against fd are exactly its
+//     goto children; flags bit k = output(first + k) != {}.  Fewer than four
+//     children repeat the last class; a state with more (or ids that do not
+//     fit) is COLD: fd = D (the ESCAPE row, all 0xFFFF) and first = 0x7FFF,
+//     so any result escapes;
+//   * states >= H are COLD.
+// A 16-bit result is 2 x + flag (x = BFS id, flag = output(x) != {}) for
+// x < 32767, and > 0xFFFD means "read the 32-bit dense table in global
+// memory (L1/L2; the paper's STT)".  Output enumeration always reads
 // that table's per-row output summary (matches are rare where this tier is
 // chosen).
 #include <algorithm>
@@ -72,22 +70,34 @@ bool split_table(ac_table &t, size_t budget) {
         for (uint32_t s = 0; s < S; s++) fd[s] = s < D ? s : fd[t.fail[s]];
     };
     // Dense levels, shallowest first: a level is made dense while most of its
-    // states would need more than two exceptions (shallow states have many
-    // children) and the level fits; then records fill the rest of the budget.
-    uint32_t D = 1;  // the root is always dense
+    // states have more than four children and the level fits; the next
+    // level gets children records.
+    auto children = [&](uint32_t s, uint32_t *cls, uint32_t *tgt, uint32_t cap) {
+        uint32_t k = 0;
+        for (uint32_t c = 0; c < C; c++) {
+            const uint32_t x = delta(s, c) & 0x7fffffffu;
+            if (t.depth[x] == t.depth[s] + 1) {  // a goto edge
+                if (k < cap) cls[k] = c, tgt[k] = delta(s, c);
+                k++;
+            }
+        }
+        return k;
+    };
+    uint32_t D = 1, d0 = 0;  // the root is always dense
     for (uint32_t d = 1; d <= maxd; d++) {
         const uint32_t lo = level_end[d - 1], hi = level_end[d];
-        if ((size_t)hi * row_bytes > budget) break;
-        set_fd(lo);
-        uint32_t over = 0, tmp[3];
-        for (uint32_t s = lo; s < hi; s++) over += exceptions(s, fd[s], tmp, 3) > 2;
+        if ((size_t)(hi + 1) * row_bytes > budget) break;
+        uint32_t over = 0, tc[5], tt[5];
+        for (uint32_t s = lo; s < hi; s++) over += children(s, tc, tt, 5) > 4;
         if (2 * over < hi - lo) break;  // mostly cheap as records
         D = hi;
+        d0 = d;
     }
-    if ((size_t)D * row_bytes > budget || D >= 0xFFFFu) return false;
+    if (D >= 4095u) return false;  // fd and the escape row index are 12-bit
     const size_t dense_bytes = (size_t)(D + 1) * row_bytes;  // + the escape row
     if (dense_bytes > budget) return false;
-    const uint32_t H = D + (uint32_t)std::min<size_t>(S - D, (budget - dense_bytes) / 8);
+    const uint32_t H = std::min<uint32_t>(level_end[d0 + 1 <= maxd ? d0 + 1 : maxd],
+                                          D + (uint32_t)std::min<size_t>(S - D, (budget - dense_bytes) / 8));
     set_fd(D);
 
     auto enc = [&](uint32_t e) -> uint16_t {  // 32-bit entry -> 2 x + flag, or the escape
@@ -105,20 +115,31 @@ bool split_table(ac_table &t, size_t budget) {
         std::memcpy(&blob[((size_t)D * dstride + c) * 2], &e, 2);
     }
     uint32_t n_cold = 0;
-    for (uint32_t s = D; s < H; s++) {  // records of the sparse hot states
-        uint32_t cls[2] = {0, 0}, lo, hi;
-        {
-            const uint32_t k = exceptions(s, fd[s], cls, 2);
-            if (k > 2) {  // cold record: every class escapes to the global table
-                lo = D;
-                hi = 0xFFFFFFFFu;
-                n_cold++;
-            } else {
-                if (k == 1) cls[1] = cls[0];
-                // k == 0: (0, delta(s, 0)) twice -- equal to the dense fallback anyway
-                lo = fd[s] | (cls[0] << 16) | (cls[1] << 24);
-                hi = (uint32_t)enc(delta(s, cls[0])) | ((uint32_t)enc(delta(s, cls[1])) << 16);
-            }
+    for (uint32_t s = D; s < H; s++) {  // children records of the next level
+        uint32_t cls[4] = {0, 0, 0, 0}, tgt[4] = {0, 0, 0, 0}, ex[1];
+        const uint32_t k = children(s, cls, tgt, 4);
+        bool ok = k <= 4 && fd[s] == t.fail[s] && exceptions(s, fd[s], ex, 0) == k;
+        for (uint32_t i = 0; ok && i < k; i++) ok = (tgt[i] & 0x7fffffffu) == (tgt[0] & 0x7fffffffu) + i;
+        ok = ok && (k == 0 || (tgt[0] & 0x7fffffffu) + k - 1 < 32767u);
+        uint32_t lo, hi;
+        if (!ok) {
+            lo = 0;
+            hi = D | (0x7FFFu << 12);  // cold: every result escapes
+            n_cold++;
+        } else if (k == 0) {
+            // a leaf: every class falls back to row[fd]; the record's class
+            // bytes (all 0) hit class 0, so "child" 0 is delta(s, 0) itself
+            const uint32_t e0 = delta(s, 0);
+            lo = 0;
+            hi = (e0 & 0x7fffffffu) < 32767u ? fd[s] | ((e0 & 0x7fffffffu) << 12) | ((e0 >> 31) << 27)
+                                             : D | (0x7FFFu << 12);
+            n_cold += (e0 & 0x7fffffffu) >= 32767u;
+        } else {
+            for (uint32_t i = k; i < 4; i++) cls[i] = cls[k - 1];  // repeats never win (lowest byte first)
+            uint32_t flags = 0;
+            for (uint32_t i = 0; i < k; i++) flags |= (tgt[i] >> 31) << i;
+            lo = cls[0] | (cls[1] << 8) | (cls[2] << 16) | (cls[3] << 24);
+            hi = fd[s] | ((tgt[0] & 0x7fffffffu) << 12) | (flags << 27);
         }
         std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8], &lo, 4);
         std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8 + 4], &hi, 4);

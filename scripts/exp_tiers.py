@@ -56,8 +56,9 @@ def main():
             cap = ac.count(stt, text) if a.exact_cap else n // 8 + 64
             out = torch.empty(max(1, cap), dtype=torch.int64, device="cuda") if a.list else None
             for v, pol in [(v, pol) for v in a.variants.split(",") for pol in a.policies.split(",")]:
-                tpol, prom = (pol + ":0").split(":")[:2]  # text policy[:promotion]
-                knobs = dict(kernel=ac.KERNEL_STAGED, variant=int(v), text_policy=int(tpol), text_promotion=int(prom))
+                tpol, prom, win = (pol + ":0:0").split(":")[:3]  # text policy[:promotion[:L2 window MiB]]
+                knobs = dict(kernel=ac.KERNEL_STAGED, variant=int(v), text_policy=int(tpol), text_promotion=int(prom),
+                             l2_window_mib=int(win))
                 try:
                     ac.match_async(stt, text, out, res, **knobs)
                 except ac.AcError as e:

@@ -285,17 +285,22 @@ def _decode_split(t):
     assert (rows[D] == 0xFFFF).all()  # the escape row
     assert blob.size == (D + 1) * ds * 2 + (H - D) * 8
     rec = blob[(D + 1) * ds * 2:].view(np.uint32).reshape(-1, 2).astype(np.int64)
-    fd = np.concatenate([np.arange(D), rec[:, 0] & 0xFFFF])  # dense states read their own row
-    no = np.full(D, 0x1FF)  # no exception class
-    c1 = np.concatenate([no, (rec[:, 0] >> 16) & 0xFF])
-    c2 = np.concatenate([no, rec[:, 0] >> 24])
-    t1 = np.concatenate([np.zeros(D, np.int64), rec[:, 1] & 0xFFFF])
-    t2 = np.concatenate([np.zeros(D, np.int64), rec[:, 1] >> 16])
-    assert (fd[D:] <= D).all()
-    cls = np.arange(C)[None, :]
-    e16 = np.where(cls == c1[:, None], t1[:, None], np.where(cls == c2[:, None], t2[:, None], rows[fd]))
+    cls4 = np.stack([(rec[:, 0] >> (8 * i)) & 0xFF for i in range(4)], axis=1)      # children's classes
+    fd = rec[:, 1] & 0xFFF
+    first = (rec[:, 1] >> 12) & 0x7FFF
+    flags = rec[:, 1] >> 27
+    assert (fd <= D).all()
+    c = np.arange(C)[None, :]
+    # first matching class byte k (lowest index) -> child first + k
+    k = np.full((H - D, C), -1, np.int64)
+    for i in range(3, -1, -1):
+        k = np.where(cls4[:, i:i + 1] == c, i, k)
+    child = ((first[:, None] + np.maximum(k, 0)) << 1) | ((flags[:, None] >> np.maximum(k, 0)) & 1)
+    e16_sparse = np.where(k >= 0, child, rows[fd])
+    e16 = np.concatenate([rows[:D], e16_sparse])
     E = (e16 >> 1) | ((e16 & 1) << 31)
-    return np.where(e16 == 0xFFFF, -1, E), int((fd[D:] == D).sum())
+    cold = (fd == D) & (first == 0x7FFF)
+    return np.where(e16 > 0xFFFD, -1, E), int(cold.sum())
 
 
 @pytest.mark.parametrize("which", ["c3", "english5k", "tiny"])
@@ -325,6 +330,7 @@ def test_split_encoding_equals_dense(which):
     # fits next to the SPLIT staged variant's ring (32 warps x 1 slot x 1 KB, 1 KB swizzle alignment)
     assert d["split_bytes"] <= 232448 - (1024 + 32 * 1024 + 256 + 16 + 256) - 128
     if which == "c3":
-        # depth <= 1 dense (root + one state per used last byte), depth-2 states as records
+        # depth <= 1 dense (root + one state per used last byte), every depth-2 state a children
+        # record, cold only with more than four children
         assert D == 1 + len({p[-1] for p in pats})
-        assert H - D >= 7000 and d["split_cold_records"] < (H - D) // 10
+        assert H - D >= 7000 and d["split_cold_records"] < (H - D) // 50
