@@ -40,12 +40,12 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
 static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
 static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)
 static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slots (32 KB ring)
-// SPLIT automata are sized for variant 10 (32 warps x 1 chain, 32-byte tiles,
-// 1 slot refilled as soon as it is copied to registers: 32 KB ring + 1 KB
-// swizzle alignment) so that both it and the lean variant 7 can stage them;
-// AUTO runs variant 7 (C3 list 1.04 vs 1.10 ms per 256 MiB; variant 10 reads
-// every text sector once -- 1.44 vs 3.3 GB of DRAM reads per GiB -- but is
-// not faster: the SPLIT scan is bound by issue and latency, not DRAM)
+// SPLIT automata run variant 10 (32 warps x 1 chain, 32-byte tiles, 1 slot
+// refilled as soon as it is copied to registers: 32 KB ring + 1 KB swizzle
+// alignment; every text sector is fetched once -- C3 list 1.44 vs 3.3 GB of
+// DRAM reads per GiB with variant 7's 16-byte boxes -- and the list step is
+// 2.5 % faster: 0.628 vs 0.644 ms per 256 MiB); they are sized so that the
+// lean variant 7 can stage them too
 static const int kSplitVariant = 10;
 // COMPACT budget used by ac_compile (no device): B200's 227 KB opt-in shared
 // memory minus the lean staged variant's ring and bookkeeping (= stt_budget)
@@ -328,7 +328,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     if (variant == 0) {
         variant = kAutoVariant;
         if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
-        if (h->tier == AC_TIER_SPLIT) variant = kLeanVariant;
+        if (h->tier == AC_TIER_SPLIT) variant = kSplitVariant;
     }
     if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, variant)) {
         set_error("staged variant " + std::to_string(variant) + " has no room for the COMPACT table");
