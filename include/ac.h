@@ -175,7 +175,7 @@ typedef struct {
     uint32_t kernel;       /* AC_KERNEL_*                                    */
     uint32_t chain_bytes;  /* bytes owned per thread chain (0 = auto; STAGED:
                               rounded to the tile width)                     */
-    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..10 (DESIGN.md
+    uint32_t variant;      /* STAGED CTA shape, 0 = auto, 1..11 (DESIGN.md
                               "Staged variants": warps x chains/lane x tile
                               width x ring depth)                            */
     uint32_t scratch_slots;/* list mode: records each chain may park in its

@@ -39,7 +39,13 @@ static ac_status cuda_fail(cudaError_t e, const char *what) {
 
 static const uint64_t kGlobalTailChain = 64;  // head/tail chains of the staged path
 static const int kAutoVariant = 4;  // 32 warps x 1 chain, 16-byte tiles, 3 slots (48 KB ring)
-static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slots (32 KB ring)
+static const int kLeanVariant = 7;  // 32 warps x 1 chain, 16-byte tiles, 2 slots (32 KB ring): sizes COMPACT
+// COMPACT automata run variant 11 (32 warps x 1 chain, one unswizzled 32-byte
+// slot copied to registers and refilled at once): C2 list 0.548 -> 0.517 ms
+// per 256 MiB (half the per-chunk ring bookkeeping per byte); its ring and
+// barriers take no more shared memory than variant 7's, so COMPACT tables
+// sized for variant 7 fit
+static const int kCompactVariant = 11;
 // SPLIT automata run variant 10 (32 warps x 1 chain, 32-byte tiles, 1 slot
 // refilled as soon as it is copied to registers: 32 KB ring + 1 KB swizzle
 // alignment; every text sector is fetched once -- C3 list 1.44 vs 3.3 GB of
@@ -327,7 +333,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     }
     if (variant == 0) {
         variant = kAutoVariant;
-        if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, kAutoVariant)) variant = kLeanVariant;
+        if (h->tier == AC_TIER_COMPACT) variant = kCompactVariant;
         if (h->tier == AC_TIER_SPLIT) variant = kSplitVariant;
     }
     if (h->tier == AC_TIER_COMPACT && h->host.compact.size() > stt_budget(h, variant)) {
@@ -1110,8 +1116,11 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
     cudaError_t e = cudaSetDevice(device);
     if (e != cudaSuccess) return fail(e, "cudaSetDevice");
     if (!t.split.empty() && tier == AC_TIER_SPLIT) {
+        // staged in 16-byte words: the padding after the blob is zeroed too
         if ((e = cudaMalloc(&h->d_split, (t.split.size() + 15) / 16 * 16)) != cudaSuccess)
             return fail(e, "cudaMalloc(split)");
+        if ((e = cudaMemset(h->d_split, 0, (t.split.size() + 15) / 16 * 16)) != cudaSuccess)
+            return fail(e, "cudaMemset(split)");
         if ((e = cudaMemcpy(h->d_split, t.split.data(), t.split.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
             return fail(e, "H2D split");
     }

@@ -158,12 +158,13 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
     const uint64_t warps = (uint64_t)gridDim.x * (blockDim.x >> 5);
     for (uint64_t c = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < n_chains; c += warps) {
         // count and end offset are loaded together (one round trip, not two);
-        // the end read for an empty chain or a tail chain is not used.
+        // the end read for an empty chain is not used.
         // (prefetching the next chain's pair during this chain's copy was
         // measured slower on C2: 0.048 -> 0.059 ms)
         const uint64_t cnt = counts[c];
-        uint64_t end = chain_end[c];
-        if (tp.tile_state && c >= tp.tail_c0) {
+        const bool tail = tp.tile_state && c >= tp.tail_c0;  // its end is not written yet: derive it
+        uint64_t end = tail ? 0 : chain_end[c];
+        if (tail) {
             // tail chain: main total + inclusive sum of the tail counts up to c
             unsigned long long v = 0;
             for (uint64_t j = tp.tail_c0 + lane; j <= c; j += 32) v += counts[j];

@@ -107,7 +107,7 @@ def test_tiers_and_widths(tier, hot, eb):
         assert_same(gpu_keys(stt, w.text, kernel=k), want)
 
 
-@pytest.mark.parametrize("variant", [0, 4, 7])
+@pytest.mark.parametrize("variant", [0, 4, 7, 11])
 @pytest.mark.parametrize("name,n,P", [("c2", 3 << 20, None), ("c1", 1 << 20, None), ("c2", 1 << 20, 60)])
 def test_compact_tier(name, n, P, variant):
     w = synth.make(name, n=n + 999, n_patterns=P)
@@ -208,7 +208,7 @@ def test_split_tier_escapes_and_cold_records():
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED), oracle_keys(o, w.text))
 
 
-@pytest.mark.parametrize("variant", [1, 3, 4, 7, 9])
+@pytest.mark.parametrize("variant", [1, 3, 4, 7, 9, 10, 11])
 def test_split_tier_variants(variant):
     # a smaller byte dictionary so the split part also fits the fat-ring variants
     w = synth.make("c3", n=(2 << 20) + 4321, n_patterns=1500)
@@ -218,7 +218,7 @@ def test_split_tier_variants(variant):
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7, 8])
+@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11])
 @pytest.mark.parametrize("name,tier", [("c1", ac.TIER_AUTO), ("c2", ac.TIER_GLOBAL), ("c2s", ac.TIER_COMPACT)])
 def test_staged_variants(variant, name, tier):
     P = {"c1": None, "c2": 400, "c2s": 80}[name]
