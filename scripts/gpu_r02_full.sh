@@ -19,7 +19,17 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 for c in c3 c2 c4; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_scan_staged -s 1 -c 1 \
     -o $O/prof_${c}_list python scripts/prof_target.py --config $c --reps 1 --mode list > $O/ncu_$c.out 2>&1
+  # gpurun copies back at most 64 MiB: keep the raw metrics as CSV, the report only for C3
+  ncu -i $O/prof_${c}_list.ncu-rep --page raw --csv > $O/prof_${c}_list.raw.csv 2>/dev/null
+  [ "$c" != "c3" ] && rm -f $O/prof_${c}_list.ncu-rep
 done
 if [ "$SKIP_SWEEP" != "1" ]; then
   timeout 2400 python scripts/sweep_c5.py --logn 28,30 --patterns 1000,5000,10000,20000,50000 > $O/sweep_c5.jsonl 2> $O/sweep_c5.err
+fi
+if [ "$WITH_SANITIZE" = "1" ]; then
+  for tool in memcheck racecheck synccheck initcheck; do
+    timeout 600 compute-sanitizer --tool $tool --target-processes all --print-limit 50 --num-cuda-barriers 128 \
+      python scripts/sanitize_target.py > $O/sanitize_$tool.log 2>&1
+    echo "exit=$?" >> $O/sanitize_$tool.log
+  done
 fi

@@ -48,7 +48,11 @@ UNITS = {
 
 
 def ncu_raw(rep: Path):
-    txt = subprocess.run(["ncu", "-i", str(rep), "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    raw = rep.with_suffix(".raw.csv")
+    if raw.exists() and raw.stat().st_size:
+        txt = raw.read_text()
+    else:
+        txt = subprocess.run(["ncu", "-i", str(rep), "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(txt.splitlines()))
     return rows[0], rows[1], rows[2:]
 
@@ -67,7 +71,9 @@ def main(tag: str = "r02"):
     PROF.mkdir(exist_ok=True)
     for src, dst in (("bench.json", f"{tag}_bench.json"), ("bench_ref.json", f"{tag}_bench_reference.json"),
                      ("pytest_gpu.log", f"{tag}_gpu_tests.log"), ("host.txt", f"{tag}_host.txt"),
-                     ("gpu.txt", f"{tag}_gpu.txt")):
+                     ("gpu.txt", f"{tag}_gpu.txt"),
+                     *[(f"sanitize_{t}.log", f"{tag}_sanitize_{t}.log")
+                       for t in ("memcheck", "racecheck", "synccheck", "initcheck")]):
         if (OUT / src).exists():
             shutil.copy(OUT / src, PROF / dst)
     if (OUT / "launches.csv").exists():
@@ -92,7 +98,7 @@ def main(tag: str = "r02"):
     traffic = {}
     for cfg in ("c3", "c2", "c4"):
         rep = OUT / f"prof_{cfg}_list.ncu-rep"
-        if not rep.exists():
+        if not rep.exists() and not rep.with_suffix(".raw.csv").exists():
             continue
         h, u, rows = ncu_raw(rep)
         r = rows[-1]
