@@ -388,6 +388,25 @@ __device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t
     }
 }
 
+// Predicated 8-byte global store to base[k] (k signed; one IMAD.WIDE for
+// the address, no branch around the store).
+__device__ __forceinline__ void st_global_if(const uint64_t *base, int32_t k, uint64_t v, bool pred) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ne.u32 p, %3, 0;\n\t"
+        "mad.wide.s32 a, %1, 8, %0;\n\t@p st.global.u64 [a], %2;\n\t}" ::"l"(base),
+        "r"(k), "l"(v), "r"((uint32_t)pred)
+        : "memory");
+}
+
+// Predicated 4-byte global store to base[k] (narrow scratch records).
+__device__ __forceinline__ void st_global32_if(const uint32_t *base, int32_t k, uint32_t v, bool pred) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ne.u32 p, %3, 0;\n\t"
+        "mad.wide.s32 a, %1, 4, %0;\n\t@p st.global.u32 [a], %2;\n\t}" ::"l"(base),
+        "r"(k), "r"(v), "r"((uint32_t)pred)
+        : "memory");
+}
+
 // One transition inside the owned chunk: count or emit output(s) at the
 // byte whose record key is key0 = (global start) << 24.  cnt is the chain's
 // running count (32-bit: the planner keeps chain_len x max|output| < 2^31).
@@ -435,6 +454,11 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
         }
         return;
     }
+    // (Dense outputs, the two-pass MODE_EMIT pass: a warp-uniform loop of
+    // max-over-lanes |output(s)| predicated loads and stores instead of this
+    // per-lane branch was measured slower -- C5 English 5K list 4.33 -> 4.72
+    // ms, 20K 2x -- the per-record dependent loads of the output CSR, not the
+    // divergence, bind that pass.)
     if (flag && live) emit_outputs<E, TIER, MODE>(s, key0, cnt, wp, s_stt, st, so);
 }
 
@@ -459,25 +483,6 @@ __device__ __forceinline__ void ac_step2(uint32_t &s, uint32_t &cnt, uint64_t &w
         if (e & T2_FIN) emit_outputs<E, TIER, MODE>(e & T2_MASK, key2, cnt, wp, s_stt, st, so);
     }
     s = e & T2_MASK;
-}
-
-// Predicated 8-byte global store to base[k] (k signed; one IMAD.WIDE for
-// the address, no branch around the store).
-__device__ __forceinline__ void st_global_if(const uint64_t *base, int32_t k, uint64_t v, bool pred) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ne.u32 p, %3, 0;\n\t"
-        "mad.wide.s32 a, %1, 8, %0;\n\t@p st.global.u64 [a], %2;\n\t}" ::"l"(base),
-        "r"(k), "l"(v), "r"((uint32_t)pred)
-        : "memory");
-}
-
-// Predicated 4-byte global store to base[k] (narrow scratch records).
-__device__ __forceinline__ void st_global32_if(const uint32_t *base, int32_t k, uint32_t v, bool pred) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t.reg .u64 a;\n\tsetp.ne.u32 p, %3, 0;\n\t"
-        "mad.wide.s32 a, %1, 4, %0;\n\t@p st.global.u32 [a], %2;\n\t}" ::"l"(base),
-        "r"(k), "r"(v), "r"((uint32_t)pred)
-        : "memory");
 }
 
 __device__ __forceinline__ uint32_t byte_of(const uint4 &v, int bb) {
