@@ -95,6 +95,20 @@ def bench_config(args, world: int) -> dict:
             "l2": "inputs larger than L2 (text >= 256 MiB per step, L2 126 MB): no flush"}
 
 
+def all_reduce(t, op=None):
+    """all_reduce in place; through host memory when the group is gloo (the
+    functional check of the N > 1 path), on the device over NCCL otherwise."""
+    import torch.distributed as dist
+    op = op if op is not None else dist.ReduceOp.SUM
+    if dist.get_backend() == "gloo" and t.is_cuda:
+        h = t.cpu()
+        dist.all_reduce(h, op=op)
+        t.copy_(h)
+    else:
+        dist.all_reduce(t, op=op)
+    return t
+
+
 def cpu_model() -> str:
     try:
         for line in Path("/proc/cpuinfo").read_text().splitlines():
@@ -277,7 +291,7 @@ def time_config(args, cfg: str, rank: int, world: int, dev, local: int, steps: i
         k = ac.match_async(stt, text, out, res, n_halo=halo, base=base, kernel=kernel)
         if world > 1:
             tot = res[:1].clone()
-            dist.all_reduce(tot)
+            all_reduce(tot)
             if out is not None:
                 allgatherv(out[:int(res[0].item())])
         return k
@@ -306,10 +320,10 @@ def time_config(args, cfg: str, rank: int, world: int, dev, local: int, steps: i
     total_owned = owned
     if world > 1:
         m = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(m, op=dist.ReduceOp.MAX)
+        all_reduce(m, op=dist.ReduceOp.MAX)
         ms = float(m.item())
         agg = torch.tensor([count, owned], dtype=torch.int64, device=dev)
-        dist.all_reduce(agg)
+        all_reduce(agg)
         total_count, total_owned = (int(x) for x in agg.tolist())
     else:
         total_count = count
@@ -384,7 +398,7 @@ def time_config(args, cfg: str, rank: int, world: int, dev, local: int, steps: i
         e_ms = s0.elapsed_time(s1) / e_steps
         if world > 1:
             m = torch.tensor([e_ms], dtype=torch.float64, device=dev)
-            dist.all_reduce(m, op=dist.ReduceOp.MAX)
+            all_reduce(m, op=dist.ReduceOp.MAX)
             e_ms = float(m.item())
         fields["e2e"] = {"value": total_owned * 8 / (e_ms * 1e-3) / 1e9, "unit": "Gbps", "h2d_bytes_per_step": owned,
                          "d2h_bytes_per_step": 16 + (8 * c_e2e if hout is not None else 0), "steps": e_steps,
@@ -402,9 +416,18 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # AC_BENCH_BACKEND=gloo: a functional check of the N > 1 path on a box
+    # with fewer GPUs than ranks (ranks share devices, collectives go through
+    # host memory); the contract run uses NCCL, one GPU per rank
+    backend = os.environ.get("AC_BENCH_BACKEND", "nccl")
+    if backend != "nccl":
+        local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     dev = torch.device("cuda", local)
     fields, w, text_np = time_config(args, args.config, rank, world, dev, local, args.steps, args.warmup, True,
                                      not args.no_e2e)

@@ -53,6 +53,13 @@ static __device__ unsigned long long ac_dbg_times[1024 * 32 * 2];
 #endif
 
 static constexpr int GT = 256;  // k_scan_global block size
+// SPLIT list mode: flag-mask walk + re-walk of flagged lanes (default) or the
+// emission inline at each flagged byte (-DAC_SPLIT_INLINE_EMIT, ablation)
+#ifdef AC_SPLIT_INLINE_EMIT
+static constexpr bool kSplitInlineEmit = true;
+#else
+static constexpr bool kSplitInlineEmit = false;
+#endif
 
 template <typename E>
 struct EntryBits;
@@ -1088,7 +1095,8 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                                                     kb[k] + ((uint64_t)bb << 24), kb[k] + ((uint64_t)(bb - 1) << 24),
                                                     live[k], s_cmap, s_stt, st, so);
                     }
-                } else if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT)) {
+                } else if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT) &&
+                                     !kSplitInlineEmit) {
                     // rare matches (the tier is chosen for large byte
                     // dictionaries): the 16 steps only collect the flag bits
                     // -- the count-mode loop, no record keys or slot
