@@ -583,3 +583,22 @@ def test_full_size_closed_form_kmers():
     d = digits.astype(np.int64)
     val = d[:-5] * 1024 + d[1:-4] * 256 + d[2:-3] * 64 + d[3:-2] * 16 + d[4:-1] * 4 + d[5:]
     assert np.array_equal(r & 0xFFFFFF, val)
+
+
+def test_cache_policy_knobs():
+    # the L2 knobs change where bytes live, never the result: text policy
+    # (normal / evict-first / per-sector pair), TMA L2 promotion, and the
+    # persisting access-policy window over the global table
+    w = synth.make("c3", n=(2 << 20) + 77)
+    o = Oracle(w.patterns)
+    want = oracle_keys(o, w.text)
+    stt = ac.build(w.patterns)
+    t = torch.from_numpy(w.text).cuda()
+    for knobs in (dict(text_policy=1), dict(text_policy=2), dict(text_policy=3), dict(text_promotion=1),
+                  dict(text_promotion=3), dict(l2_window_mib=16), dict(l2_window_mib=64, text_policy=1)):
+        c, recs = ac.match(stt, t, kernel=ac.KERNEL_STAGED, **knobs)
+        assert_same(recs.cpu().numpy(), want)
+    res = torch.zeros(2, dtype=torch.int64, device="cuda")
+    for bad in (dict(text_policy=4), dict(text_promotion=5)):
+        with pytest.raises(ac.AcError):
+            ac.match_async(stt, t, None, res, **bad)
