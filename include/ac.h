@@ -110,6 +110,10 @@ typedef struct {
                               <= 8 classes whose two-byte table fits 64 MiB),
                               1, or 2 (needs 32-bit
                               entries -- set entry_bytes = 4 for small S)    */
+    uint32_t threads;      /* host threads for phase 1:
+                              0 = $AC_BUILD_THREADS if set, else the
+                              hardware concurrency (at most 32); the table
+                              is identical for every value                  */
 } ac_build_opts;
 
 typedef struct {

@@ -52,7 +52,8 @@ class CapacityError(AcError):
 
 class ac_build_opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_uint32), ("entry_bytes", ctypes.c_uint32), ("tier", ctypes.c_uint32),
-                ("hot_rows", ctypes.c_uint32), ("forward", ctypes.c_uint32), ("stride", ctypes.c_uint32)]
+                ("hot_rows", ctypes.c_uint32), ("forward", ctypes.c_uint32), ("stride", ctypes.c_uint32),
+                ("threads", ctypes.c_uint32)]
 
 
 class ac_stt_info(ctypes.Structure):
@@ -151,8 +152,9 @@ def _pattern_arrays(patterns):
     return pats, bufs, ptrs, lens
 
 
-def _opts(entry_bytes=0, tier=TIER_AUTO, hot_rows=0, forward=False, stride=0):
-    return ac_build_opts(ctypes.sizeof(ac_build_opts), entry_bytes, tier, hot_rows, 1 if forward else 0, stride)
+def _opts(entry_bytes=0, tier=TIER_AUTO, hot_rows=0, forward=False, stride=0, threads=0):
+    return ac_build_opts(ctypes.sizeof(ac_build_opts), entry_bytes, tier, hot_rows, 1 if forward else 0, stride,
+                         threads)
 
 
 def _info_dict(info: ac_stt_info) -> dict:
@@ -163,11 +165,11 @@ class Stt:
     """A device STT (phase-1 result), immutable, freed with the object."""
 
     def __init__(self, patterns, device: int = 0, entry_bytes: int = 0, tier: int = TIER_AUTO, hot_rows: int = 0,
-                 stride: int = 0):
+                 stride: int = 0, threads: int = 0):
         L = lib()
         self.patterns, bufs, ptrs, lens = _pattern_arrays(patterns)
         h = ctypes.c_void_p()
-        o = _opts(entry_bytes, tier, hot_rows, stride=stride)
+        o = _opts(entry_bytes, tier, hot_rows, stride=stride, threads=threads)
         _check(L.ac_build(ptrs, lens, len(self.patterns), int(device), ctypes.byref(o), ctypes.byref(h)))
         self._h = h
         self.device = int(device)
@@ -374,14 +376,14 @@ class HostTable:
 
 
 def compile_table(patterns, forward: bool = False, entry_bytes: int = 0, compact: bool = False,
-                  stride: int = 0, split: bool = False) -> HostTable:
+                  stride: int = 0, split: bool = False, threads: int = 0) -> HostTable:
     """Phase 1 on the host only (no device) -- for builder tests."""
     import numpy as np
     L = lib()
     pats, bufs, ptrs, lens = _pattern_arrays(patterns)
     h = ctypes.c_void_p()
     tier = TIER_COMPACT if compact else TIER_SPLIT if split else TIER_AUTO
-    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=tier, stride=stride)
+    o = _opts(entry_bytes=entry_bytes, forward=forward, tier=tier, stride=stride, threads=threads)
     _check(L.ac_compile(ptrs, lens, len(pats), ctypes.byref(o), ctypes.byref(h)))
     try:
         info = ac_stt_info()

@@ -1029,7 +1029,7 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
         ac_table t4;
         ac_table *ts = &h->host;
         if (t.entry_bytes != 4) {
-            ac_build_opts o = opts ? *opts : ac_build_opts{sizeof(ac_build_opts), 0, 0, 0, 0, 0};
+            ac_build_opts o = opts ? *opts : ac_build_opts{sizeof(ac_build_opts), 0, 0, 0, 0, 0, 0};
             o.entry_bytes = 4;
             try {
                 rc = compile_table(patterns, lens, n, &o, t4);

@@ -23,15 +23,46 @@
 //   * output(s) is stored as CSR with ids ascending (the closure over the
 //     failure function).
 //
-// Construction is the textbook one (AC'75 Alg. 2-4) on a dense goto table.
+// Construction is the textbook one (AC'75 Alg. 2-4) on a dense goto table;
+// everything after the trie runs on host threads, one BFS level at a time
+// (a faster build).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
-#include <deque>
 #include <new>
+#include <thread>
 
 #include "ac_internal.h"
 
 namespace acx {
+
+// Host threads for phase 1: ac_build_opts.threads, else $AC_BUILD_THREADS,
+// else the hardware concurrency (capped at 32).
+uint32_t build_threads(const ac_build_opts *opts) {
+    uint32_t t = opts ? opts->threads : 0;
+    if (t == 0) {
+        const char *e = std::getenv("AC_BUILD_THREADS");
+        if (e && *e) t = (uint32_t)std::strtoul(e, nullptr, 10);
+    }
+    if (t == 0) t = std::min(32u, std::max(1u, std::thread::hardware_concurrency()));
+    return std::max(1u, std::min(t, 256u));
+}
+
+// fn(lo, hi) over [0, n) in T contiguous ranges; small ranges stay on the
+// calling thread (a level of a few hundred states is not worth a spawn).
+void parallel_for(size_t n, uint32_t T, const std::function<void(size_t, size_t)> &fn) {
+    const size_t kMinPerThread = 2048;
+    size_t k = std::min<size_t>(T, (n + kMinPerThread - 1) / kMinPerThread);
+    if (k <= 1) {
+        if (n) fn(0, n);
+        return;
+    }
+    std::vector<std::thread> pool;
+    pool.reserve(k - 1);
+    for (size_t j = 1; j < k; j++) pool.emplace_back(fn, n * j / k, n * (j + 1) / k);
+    fn(0, n / k);
+    for (auto &th : pool) th.join();
+}
 
 ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n,
                         const ac_build_opts *opts, ac_table &t) {
@@ -86,12 +117,17 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
     }
     t.n_classes = C;
 
+    const uint32_t T = build_threads(opts);
     try {
-        // ---- goto function (AC'75 Alg. 2) on a dense table, creation order
+        // ---- goto function (AC'75 Alg. 2) on a dense table, creation order.
+        // The trie is sequential (one pass over the patterns); every later
+        // phase runs on T threads, level by level where a state depends on
+        // shallower ones (NEXT-3 "faster build"; the table is identical for
+        // any T).
         std::vector<int32_t> go;
         go.reserve((size_t)std::min<uint64_t>(total + 1, 1u << 22) * C);
         go.assign(C, -1);
-        std::vector<std::vector<uint32_t>> own(1);
+        std::vector<uint32_t> end_state(n);
         uint32_t S = 1;
         for (uint32_t p = 0; p < n; p++) {
             uint32_t s = 0;
@@ -103,56 +139,86 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
                     nx = (int32_t)S++;
                     go[(size_t)s * C + c] = nx;
                     go.insert(go.end(), C, -1);
-                    own.emplace_back();
                 }
                 s = (uint32_t)nx;
             }
-            own[s].push_back(p);
+            end_state[p] = s;
         }
-        // ---- BFS order, failure function and delta (AC'75 Alg. 3/4)
+        // own(s): the patterns ending in s, ids ascending (counting sort)
+        std::vector<uint32_t> own_off(S + 1, 0), own_ids(n);
+        for (uint32_t p = 0; p < n; p++) own_off[end_state[p] + 1]++;
+        for (uint32_t s = 0; s < S; s++) own_off[s + 1] += own_off[s];
+        {
+            std::vector<uint32_t> fill(own_off.begin(), own_off.end() - 1);
+            for (uint32_t p = 0; p < n; p++) own_ids[fill[end_state[p]]++] = p;
+        }
+        // ---- BFS order, failure function and delta (AC'75 Alg. 3/4), one
+        // level at a time: a state's failure state is shallower, so its delta
+        // row is final before the level that reads it.
         std::vector<uint32_t> order;
         order.reserve(S);
-        std::vector<uint32_t> fail(S, 0), depth(S, 0);
+        std::vector<uint32_t> fail(S, 0), depth(S, 0), level_start;
         order.push_back(0);
-        for (size_t qi = 0; qi < order.size(); qi++) {
-            uint32_t r = order[qi];
-            int32_t *row = &go[(size_t)r * C];
-            for (uint32_t c = 0; c < C; c++) {
-                int32_t child = row[c];
-                if (child >= 0) {
-                    order.push_back((uint32_t)child);
-                    depth[child] = depth[r] + 1;
-                    fail[child] = (r == 0) ? 0u : (uint32_t)(go[(size_t)fail[r] * C + c] & 0x7fffffff);
-                    row[c] = child;
-                } else {
-                    // delta(r,c) = delta(f(r),c); the root loops to itself
-                    row[c] = (r == 0) ? 0 : go[(size_t)fail[r] * C + c];
+        std::vector<uint32_t> nch;
+        for (size_t lo = 0, hi = 1; lo < hi; lo = hi, hi = order.size()) {
+            level_start.push_back((uint32_t)lo);
+            const size_t L = hi - lo;
+            nch.assign(L + 1, 0);
+            parallel_for(L, T, [&](size_t a, size_t b) {
+                for (size_t i = a; i < b; i++) {
+                    const int32_t *row = &go[(size_t)order[lo + i] * C];
+                    uint32_t k = 0;
+                    for (uint32_t c = 0; c < C; c++) k += row[c] >= 0;
+                    nch[i + 1] = k;
                 }
-            }
+            });
+            for (size_t i = 0; i < L; i++) nch[i + 1] += nch[i];
+            order.resize(hi + nch[L]);
+            parallel_for(L, T, [&](size_t a, size_t b) {
+                for (size_t i = a; i < b; i++) {
+                    const uint32_t r = order[lo + i];
+                    int32_t *row = &go[(size_t)r * C];
+                    const int32_t *frow = &go[(size_t)fail[r] * C];
+                    size_t w = hi + nch[i];
+                    for (uint32_t c = 0; c < C; c++) {
+                        const int32_t child = row[c];
+                        if (child >= 0) {
+                            order[w++] = (uint32_t)child;
+                            depth[child] = depth[r] + 1;
+                            fail[child] = (r == 0) ? 0u : (uint32_t)frow[c];
+                        } else {
+                            // delta(r,c) = delta(f(r),c); the root loops to itself
+                            row[c] = (r == 0) ? 0 : frow[c];
+                        }
+                    }
+                }
+            });
         }
+        level_start.push_back(S);
         // after this loop go[] holds delta (all entries >= 0)
-        // ---- output closure, in BFS order (f(s) is shallower than s)
-        std::vector<std::vector<uint32_t>> out(S);
-        for (uint32_t s : order) {
-            std::vector<uint32_t> v = own[s];
-            if (s != 0) {
-                const std::vector<uint32_t> &fo = out[fail[s]];
-                v.insert(v.end(), fo.begin(), fo.end());
-            }
-            std::sort(v.begin(), v.end());
-            out[s].swap(v);
-        }
-        own.clear();
-        own.shrink_to_fit();
         // ---- renumber in BFS order
         std::vector<uint32_t> rank(S);
-        for (uint32_t i = 0; i < S; i++) rank[order[i]] = i;
+        parallel_for(S, T, [&](size_t a, size_t b) {
+            for (size_t i = a; i < b; i++) rank[order[i]] = (uint32_t)i;
+        });
         t.fail.resize(S);
         t.depth.resize(S);
-        for (uint32_t i = 0; i < S; i++) {
-            t.fail[i] = rank[fail[order[i]]];
-            t.depth[i] = depth[order[i]];
-        }
+        parallel_for(S, T, [&](size_t a, size_t b) {
+            for (size_t i = a; i < b; i++) {
+                t.fail[i] = rank[fail[order[i]]];
+                t.depth[i] = depth[order[i]];
+            }
+        });
+        // ---- output closure output(s) = own(s) U output(f(s)),
+        // as CSR in BFS numbering; |output(s)| and the fill go level by level
+        std::vector<uint64_t> osz(S, 0);  // by BFS id
+        for (size_t d = 0; d + 1 < level_start.size(); d++)
+            parallel_for(level_start[d + 1] - level_start[d], T, [&](size_t a, size_t b) {
+                for (size_t i = level_start[d] + a; i < level_start[d] + b; i++) {
+                    const uint32_t s = order[i];
+                    osz[i] = (own_off[s + 1] - own_off[s]) + (i ? osz[rank[fail[s]]] : 0);
+                }
+            });
         uint32_t eb = want_eb ? want_eb : (S <= 32768 ? 2u : 4u);
         if (eb == 2 && S > 32768) {
             set_error("entry_bytes=2 needs <= 32768 states");
@@ -179,14 +245,13 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
         t.row_stride = stride;
         t.info_col = info_col;
         t.entry_bytes = eb;
-        t.stt.assign((size_t)S * stride * eb, 0);
         t.out_off.assign(S + 1, 0);
         uint64_t n_out = 0;
         t.max_out = 0;
         for (uint32_t i = 0; i < S; i++) {
             t.out_off[i] = (uint32_t)n_out;
-            n_out += out[order[i]].size();
-            t.max_out = std::max<uint32_t>(t.max_out, (uint32_t)out[order[i]].size());
+            n_out += osz[i];
+            t.max_out = (uint32_t)std::max<uint64_t>(t.max_out, osz[i]);
             if (n_out >= (1ull << 32)) {
                 set_error("output closure too large");
                 return AC_ERR_TOO_LARGE;
@@ -194,35 +259,47 @@ ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, ui
         }
         t.out_off[S] = (uint32_t)n_out;
         t.out_ids.resize(n_out);
-        for (uint32_t i = 0; i < S; i++) {
-            const std::vector<uint32_t> &v = out[order[i]];
-            std::copy(v.begin(), v.end(), t.out_ids.begin() + t.out_off[i]);
-        }
-        for (uint32_t i = 0; i < S; i++) {
-            const int32_t *row = &go[(size_t)order[i] * C];
-            const std::vector<uint32_t> &v = out[order[i]];
-            const uint32_t payload = v.size() == 1 ? v[0] : t.out_off[i];
-            uint8_t *r = &t.stt[(size_t)i * stride * eb];
-            std::memcpy(r + (size_t)info_col * eb, &payload, 4);
-            if (eb == 2) {
-                uint16_t c16 = (uint16_t)std::min<size_t>(v.size(), 0xFFFF);
-                std::memcpy(r + (size_t)(info_col + 2) * 2, &c16, 2);
-            } else {
-                uint32_t c32 = (uint32_t)v.size();
-                std::memcpy(r + (size_t)(info_col + 1) * 4, &c32, 4);
-            }
-            for (uint32_t c = 0; c < C; c++) {
-                uint32_t nx = rank[(uint32_t)row[c]];
-                bool flag = !out[(uint32_t)row[c]].empty();
+        for (size_t d = 0; d + 1 < level_start.size(); d++)
+            parallel_for(level_start[d + 1] - level_start[d], T, [&](size_t a, size_t b) {
+                for (size_t i = level_start[d] + a; i < level_start[d] + b; i++) {
+                    const uint32_t s = order[i];
+                    uint32_t *dst = t.out_ids.data() + t.out_off[i];
+                    if (i == 0) {
+                        std::copy(own_ids.begin() + own_off[s], own_ids.begin() + own_off[s + 1], dst);
+                    } else {
+                        const uint32_t f = rank[fail[s]];  // shallower: already filled
+                        std::merge(own_ids.begin() + own_off[s], own_ids.begin() + own_off[s + 1],
+                                   t.out_ids.begin() + t.out_off[f], t.out_ids.begin() + t.out_off[f + 1], dst);
+                    }
+                }
+            });
+        // ---- the table: entry = BFS id of delta(s,c) | flag (output non-empty)
+        std::vector<uint32_t> code(S);  // by creation id
+        parallel_for(S, T, [&](size_t a, size_t b) {
+            for (size_t s = a; s < b; s++)
+                code[s] = rank[s] | (osz[rank[s]] ? (eb == 2 ? 0x8000u : 0x80000000u) : 0u);
+        });
+        t.stt.assign((size_t)S * stride * eb, 0);
+        parallel_for(S, T, [&](size_t a, size_t b) {
+            for (size_t i = a; i < b; i++) {
+                const int32_t *row = &go[(size_t)order[i] * C];
+                const uint64_t cnt = osz[i];
+                const uint32_t payload = cnt == 1 ? t.out_ids[t.out_off[i]] : t.out_off[i];
+                uint8_t *r = &t.stt[(size_t)i * stride * eb];
+                std::memcpy(r + (size_t)info_col * eb, &payload, 4);
                 if (eb == 2) {
-                    uint16_t e = (uint16_t)(nx | (flag ? 0x8000u : 0u));
-                    std::memcpy(&t.stt[((size_t)i * stride + c) * 2], &e, 2);
+                    uint16_t c16 = (uint16_t)std::min<uint64_t>(cnt, 0xFFFF);
+                    std::memcpy(r + (size_t)(info_col + 2) * 2, &c16, 2);
+                    uint16_t *e = reinterpret_cast<uint16_t *>(r);
+                    for (uint32_t c = 0; c < C; c++) e[c] = (uint16_t)code[(uint32_t)row[c]];
                 } else {
-                    uint32_t e = nx | (flag ? 0x80000000u : 0u);
-                    std::memcpy(&t.stt[((size_t)i * stride + c) * 4], &e, 4);
+                    uint32_t c32 = (uint32_t)cnt;
+                    std::memcpy(r + (size_t)(info_col + 1) * 4, &c32, 4);
+                    uint32_t *e = reinterpret_cast<uint32_t *>(r);
+                    for (uint32_t c = 0; c < C; c++) e[c] = code[(uint32_t)row[c]];
                 }
             }
-        }
+        });
     } catch (const std::bad_alloc &) {
         set_error("host allocation failed while building the STT");
         return AC_ERR_NO_MEMORY;

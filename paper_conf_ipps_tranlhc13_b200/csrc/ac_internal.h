@@ -2,6 +2,7 @@
 #pragma once
 
 #include <cstdint>
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -68,6 +69,8 @@ struct ac_stt {
 
 namespace acx {
 void set_error(const std::string &msg);
+uint32_t build_threads(const ac_build_opts *opts);
+void parallel_for(size_t n, uint32_t T, const std::function<void(size_t, size_t)> &fn);
 ac_status compile_table(const uint8_t *const *patterns, const uint32_t *lens, uint32_t n,
                         const ac_build_opts *opts, ac_table &t);
 bool compact_table(ac_table &t, size_t budget);
