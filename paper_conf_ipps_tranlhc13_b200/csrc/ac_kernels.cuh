@@ -469,6 +469,76 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
     if (flag && live) emit_outputs<E, TIER, MODE>(s, key0, cnt, wp, s_stt, st, so);
 }
 
+// Two-pass emission (MODE_EMIT) from a CONVERGED warp -- the staged scan's
+// per-byte and per-chunk loops only (a full-mask vote in the divergent
+// callers, halo warm-ups and re-walks, would deadlock).  f = this lane
+// reaches output state x at key0.  A single-output state's record is stored
+// by its own lane; the records of a multi-output state are written by the
+// whole warp, one such lane at a time: 32 consecutive ids read and 32
+// consecutive records written per instruction.  Per-lane loops cost one
+// L1 wavefront per record for the id and another for the store (each lane
+// writes its own chain's range: 32 lines per instruction), which is what
+// bound dense dictionaries (C5 English: 4-14 outputs per flagged byte).
+#ifndef AC_COOP_MIN
+#define AC_COOP_MIN 2  // smallest |output(x)| written by the whole warp
+#endif
+#ifndef AC_COOP_BATCH
+#define AC_COOP_BATCH 1  // multi-output states whose id loads are in flight together
+#endif
+#ifndef AC_COOP
+#define AC_COOP 1  // 0: per-lane emission in the two-pass MODE_EMIT loops (ablation)
+#endif
+template <typename E, int TIER>
+__device__ __forceinline__ void emit_coop(uint32_t x, uint32_t f, uint64_t key0, uint64_t &wp, const E *s_stt,
+                                          const SttView &st, const ScanOut &so) {
+    if (!__any_sync(0xffffffffu, f)) return;
+    const uint2 o = out_info_pred<E, TIER, true>(s_stt, st, x, f);
+    uint32_t c = o.y;
+    if (TIER != AC_TIER_COMPACT && sizeof(E) == 2 && c == 0xFFFFu)
+        c = __ldg(st.out_off + x + 1) - __ldg(st.out_off + x);
+    const bool coop = c >= (uint32_t)AC_COOP_MIN;
+    if (!coop) {  // one lane, few records
+        if (c == 1u) {
+            so.out[--wp] = key0 | o.x;
+        } else {
+            for (uint32_t j = o.x + c; j > o.x; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
+        }
+    }
+    uint32_t multi = __ballot_sync(0xffffffffu, coop);
+    const uint32_t lane = threadIdx.x & 31u;
+    while (multi) {
+        // up to AC_COOP_BATCH states: their (count, payload, key, first
+        // record) broadcast, then every id load issued before any store
+        uint32_t cc[AC_COOP_BATCH], pp[AC_COOP_BATCH];
+        uint64_t kk[AC_COOP_BATCH], dd[AC_COOP_BATCH];
+        uint32_t big = 0;
+#pragma unroll
+        for (int u = 0; u < AC_COOP_BATCH; u++) {
+            const int i = multi ? __ffs(multi) - 1 : 0;
+            const uint32_t has = multi != 0;
+            multi &= multi - 1u;
+            cc[u] = __shfl_sync(0xffffffffu, c, i) * has;
+            pp[u] = __shfl_sync(0xffffffffu, o.x, i);
+            kk[u] = __shfl_sync(0xffffffffu, key0, i);
+            dd[u] = __shfl_sync(0xffffffffu, wp, i) - cc[u];
+            big |= cc[u] > 32u;
+        }
+        if (!big) {
+            uint32_t id[AC_COOP_BATCH];
+#pragma unroll
+            for (int u = 0; u < AC_COOP_BATCH; u++) id[u] = lane < cc[u] ? __ldg(st.out_ids + pp[u] + lane) : 0u;
+#pragma unroll
+            for (int u = 0; u < AC_COOP_BATCH; u++)
+                if (lane < cc[u]) so.out[dd[u] + lane] = kk[u] | id[u];
+        } else {
+#pragma unroll
+            for (int u = 0; u < AC_COOP_BATCH; u++)
+                for (uint32_t b = lane; b < cc[u]; b += 32u) so.out[dd[u] + b] = kk[u] | __ldg(st.out_ids + pp[u] + b);
+        }
+    }
+    if (coop) wp -= c;
+}
+
 // NEXT-4: one lookup for two bytes.  T2[s][c1*C + c2] =
 // delta(delta(s,c1),c2) with bit 31 = output(final) != {} and bit 30 =
 // output(middle) != {}; the (rare) middle state is recovered from the
@@ -1071,6 +1141,22 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                         else
                             emit_loop(std::false_type{});
                         cnt[0] = (uint32_t)(-nk);
+                    } else if constexpr (MODE == MODE_EMIT && AC_COOP) {
+                        // two-pass emission (dense outputs): one flagged byte
+                        // per lane per round, multi-output states written by
+                        // the whole warp (emit_coop)
+                        while (__any_sync(0xffffffffu, fm)) {
+                            const uint32_t act = fm != 0;
+                            const int bb = act ? 31 - __clz(fm) : 0;
+                            fm &= ~(act << bb);
+                            const int i = bb >> 1;
+                            const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
+                            const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
+                            const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
+                            const uint32_t pr = (i & 4) ? b1 : b0;
+                            const uint32_t x = (bb & 1) ? (pr & 0xFFFFu) : (pr >> 16);
+                            emit_coop<E, TIER>(x, act, kb[0] + ((uint64_t)bb << 24), wp[0], s_stt, st, so);
+                        }
                     } else
                     while (__any_sync(0xffffffffu, fm)) {
                         if (fm) {
@@ -1114,7 +1200,23 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                             s[k] = state_of<E, TIER>(e, st);
                             fm |= flag_of<E, TIER>(e, s[k], st) << bb;
                         }
-                        if (__any_sync(0xffffffffu, fm != 0 && live[k]) && fm != 0 && live[k]) {
+                        if constexpr (MODE == MODE_EMIT && AC_COOP) {
+                            // two-pass emission (dense outputs): every lane
+                            // re-walks in step so the warp can write the
+                            // multi-output states' records together (emit_coop)
+                            if (!live[k]) fm = 0;
+                            if (__any_sync(0xffffffffu, fm != 0)) {
+                                uint32_t x = s_in;
+#pragma unroll 1
+                                for (int bb = 15; bb >= 0; --bb) {
+                                    const uint32_t e = next_entry<E, TIER>(
+                                        s_stt, st, x, class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                                    x = state_of<E, TIER>(e, st);
+                                    emit_coop<E, TIER>(x, (fm >> bb) & 1u, kb[k] + ((uint64_t)bb << 24), wp[k], s_stt,
+                                                       st, so);
+                                }
+                            }
+                        } else if (__any_sync(0xffffffffu, fm != 0 && live[k]) && fm != 0 && live[k]) {
                             uint32_t x = s_in;
 #pragma unroll 1
                             for (int bb = 15; bb >= 0; --bb) {
@@ -1139,6 +1241,19 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                             if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k])
                                 emit_outputs<E, TIER, MODE>(s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
                                                             st, so);
+                        }
+                    }
+                } else if constexpr (MODE == MODE_EMIT && AC_COOP) {
+                    // two-pass emission (dense outputs), warp-cooperative
+#pragma unroll
+                    for (int bb = 15; bb >= 0; --bb) {
+#pragma unroll
+                        for (int k = 0; k < K; k++) {
+                            const uint32_t e = next_entry<E, TIER>(s_stt, st, s[k],
+                                                                   class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                            s[k] = state_of<E, TIER>(e, st);
+                            const uint32_t f = flag_of<E, TIER>(e, s[k], st) & (live[k] ? 1u : 0u);
+                            emit_coop<E, TIER>(s[k], f, kb[k] + ((uint64_t)bb << 24), wp[k], s_stt, st, so);
                         }
                     }
                 } else {

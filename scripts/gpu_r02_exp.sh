@@ -1,11 +1,14 @@
 #!/bin/bash
-mkdir -p gpurun_out/exp
-python -c "import __graft_entry__ as g; g.build()" > gpurun_out/exp/build.log 2>&1
-for r in 1 2; do
-timeout 300 python scripts/exp_tiers.py --workloads c3 --tiers split --variants 0 --list >> gpurun_out/exp/tiers_rewalk.jsonl 2>> gpurun_out/exp/tiers.err
+# scratch recipe for the current experiment: emit_coop on/off/batch x staged variants
+O=gpurun_out/exp4
+mkdir -p $O
+LIB=paper_conf_ipps_tranlhc13_b200/libac.so
+for v in coop_b1 coop0 coop_b2; do
+  cp exp_libs/$v.so $LIB
+  timeout 600 python scripts/exp_tiers.py --workloads c5-english-5000-28 --tiers auto --list --exact-cap --variants 0,1,5,9,12 2>> $O/tiers.err | sed "s/^{/{\"lib\": \"$v\", /" >> $O/tiers.jsonl
+  timeout 600 python scripts/exp_tiers.py --workloads c5-english-20000-28 --tiers auto --list --exact-cap --variants 0,12 2>> $O/tiers.err | sed "s/^{/{\"lib\": \"$v\", /" >> $O/tiers.jsonl
 done
-AC_EXTRA_NVCC_FLAGS=-DAC_SPLIT_INLINE_EMIT python -c "
-from paper_conf_ipps_tranlhc13_b200 import _build; _build.build(force=True)" > gpurun_out/exp/build2.log 2>&1
-for r in 1 2; do
-timeout 300 python scripts/exp_tiers.py --workloads c3 --tiers split --variants 0 --list >> gpurun_out/exp/tiers_inline.jsonl 2>> gpurun_out/exp/tiers.err
-done
+cp exp_libs/coop_b1.so $LIB
+timeout 600 python scripts/exp_tiers.py --workloads c3,c2 --tiers auto --list --variants 0,12 2>> $O/tiers.err | sed "s/^{/{\"lib\": \"coop_b1\", /" >> $O/tiers.jsonl
+timeout 600 python scripts/exp_tiers.py --workloads c3 --tiers auto --variants 0,12 2>> $O/tiers.err | sed "s/^{/{\"lib\": \"coop_b1\", /" >> $O/tiers.jsonl
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "variants or split" > $O/pytest.log 2>&1; echo "rc=$?" >> $O/pytest.log

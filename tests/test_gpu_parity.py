@@ -125,6 +125,23 @@ def test_compact_tier(name, n, P, variant):
         assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_GLOBAL), want)
 
 
+@pytest.mark.parametrize("P,tier", [(1000, ac.TIER_AUTO), (5000, ac.TIER_AUTO), (5000, ac.TIER_SPLIT),
+                                    (20000, ac.TIER_AUTO), (20000, ac.TIER_GLOBAL)])
+def test_dense_outputs_english(P, tier):
+    """C5 English dictionaries: 0.26-5.2 matches per byte, up to 78 patterns
+    per output state -- the two-pass emission with the warp-cooperative
+    writes of multi-output states (emit_coop) in every tier the family lands
+    in (COMPACT 1K, GLOBAL 5K, SPLIT 20K), record by record."""
+    voc = synth.english_vocabulary(5002)
+    text = synth.text_english((2 << 20) + 4321, 5000, voc)
+    pats = synth.patterns_substrings(text, P, 4, 32, 5001)
+    o = Oracle(pats)
+    stt = ac.build(pats, tier=tier)
+    want = oracle_keys(o, text)
+    assert want.size > text.size // 5
+    assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED), want)
+
+
 def test_compact_is_auto_for_c2():
     w = synth.make("c2", n=1 << 20)
     stt = ac.build(w.patterns)
@@ -208,7 +225,7 @@ def test_split_tier_escapes_and_cold_records():
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED), oracle_keys(o, w.text))
 
 
-@pytest.mark.parametrize("variant", [1, 3, 4, 7, 9, 10, 11])
+@pytest.mark.parametrize("variant", [1, 3, 4, 7, 9, 10, 11, 12])
 def test_split_tier_variants(variant):
     # a smaller byte dictionary so the split part also fits the fat-ring variants
     w = synth.make("c3", n=(2 << 20) + 4321, n_patterns=1500)
@@ -218,7 +235,7 @@ def test_split_tier_variants(variant):
     assert_same(gpu_keys(stt, w.text, kernel=ac.KERNEL_STAGED, variant=variant), want)
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11])
+@pytest.mark.parametrize("variant", [1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11, 12])
 @pytest.mark.parametrize("name,tier", [("c1", ac.TIER_AUTO), ("c2", ac.TIER_GLOBAL), ("c2s", ac.TIER_COMPACT)])
 def test_staged_variants(variant, name, tier):
     P = {"c1": None, "c2": 400, "c2s": 80}[name]
@@ -508,6 +525,45 @@ def digest_keys(keys: np.ndarray):
             sm = (sm + int(h.sum(dtype=np.uint64))) & ((1 << 64) - 1)
         x ^= int(np.bitwise_xor.reduce(h)) if h.size else 0
     return c, sm, x
+
+
+def _s64(c: int) -> int:
+    return c - (1 << 64) if c >= 1 << 63 else c
+
+
+def _torch_mix64(z: torch.Tensor) -> torch.Tensor:
+    """splitmix64 over an int64 tensor (two's-complement wrapping = uint64
+    arithmetic; logical shifts by masking the arithmetic ones)."""
+    def shr(v, k):
+        return (v >> k) & ((1 << (64 - k)) - 1)
+    z = z + _s64(0x9E3779B97F4A7C15)
+    z = (z ^ shr(z, 30)) * _s64(0xBF58476D1CE4E5B9)
+    z = (z ^ shr(z, 27)) * _s64(0x94D049BB133111EB)
+    return z ^ shr(z, 31)
+
+
+def digest_keys_torch(keys: torch.Tensor, chunk: int = 1 << 27):
+    """digest_keys on the device (test side, for lists too large to copy to
+    the host): the same (count, sum mod 2^64, xor) of splitmix64."""
+    k = keys.reshape(-1)
+    sm, x = 0, 0
+    for lo in range(0, k.numel(), chunk):
+        h = _torch_mix64(k[lo:lo + chunk])
+        sm = (sm + int(h.sum()) % (1 << 64)) % (1 << 64)
+        while h.numel() > 1:
+            if h.numel() & 1:  # fold the odd element into the first
+                h = torch.cat([h[:1] ^ h[-1:], h[1:-1]])
+            half = h.numel() // 2
+            h = h[:half] ^ h[half:]
+        x ^= int(h[0]) % (1 << 64) if h.numel() else 0
+    return int(k.numel()), sm, x
+
+
+def test_torch_digest_matches_numpy():
+    rng = np.random.default_rng(3)
+    for n in (0, 1, 7, 1000, (1 << 20) + 3):
+        a = rng.integers(0, 1 << 62, size=n, dtype=np.int64) << 1
+        assert digest_keys_torch(torch.from_numpy(a).cuda(), chunk=1 << 18) == digest_keys(a)
 
 
 def test_np_mix64_known_values():
