@@ -167,7 +167,8 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
 __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
     const uint32_t rep = cls * 0x01010101u;
     const uint32_t sparse = (s - st.s_dense) < (st.s_rec - st.s_dense);
-    uint32_t lo = base + st.s_rec_x0 + s * 8u;  // record address (biased by -8 s_dense)
+    const uint32_t rbase = base + st.s_rec_x0;  // loop-invariant: one uniform register
+    uint32_t lo = rbase + s * 8u;               // record address (biased by -8 s_dense)
     uint32_t hi = min(s, st.s_dense);           // fd of a dense state (itself) or of a cold one (escape row)
     asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%0];\n\t"
         "@!p xor.b32 %0, %3, 0x80808080;\n\t}"
@@ -177,12 +178,13 @@ __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st,
     const uint32_t x = lo ^ rep;                                  // a zero byte where a class matches
     const uint32_t z = (x - 0x01010101u) & ~x & 0x80808080u;      // lowest set bit: the first match
     const uint32_t kk = (__ffs(z) - 1u) >> 3;                      // child index (garbage if no match)
-    uint32_t e = base + (hi & 0xFFFu) * st.s_row_bytes + cls * 2u;  // row[fd][cls]
-    asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t}"
-        : "+r"(e)
-        : "r"(z));
     const uint32_t child = ((((hi >> 12) & 0x7FFFu) + kk) << 1) | ((hi >> (27u + kk)) & 1u);
-    const uint32_t e16 = z ? child : e;
+    // e16 = child if a class matched, else the shared row entry row[fd][cls]:
+    // one predicate for the load and the select
+    uint32_t e16 = base + (hi & 0xFFFu) * st.s_row_bytes + cls * 2u;
+    asm("{\n\t.reg .pred p;\n\tsetp.eq.u32 p, %1, 0;\n\t@p ld.shared.u16 %0, [%0];\n\t@!p mov.b32 %0, %2;\n\t}"
+        : "+r"(e16)
+        : "r"(z), "r"(child));
     uint32_t g = (e16 >> 1) | (e16 << 31);  // 2 x + flag -> x | flag << 31
     // (a warp-uniform skip of this block -- a vote over the active lanes --
     // was measured slower than the predicated form: C3 count 0.48 -> 0.51 ms,
@@ -469,24 +471,29 @@ __device__ __forceinline__ void ac_step(uint32_t &s, uint32_t &cnt, uint64_t &wp
     if (flag && live) emit_outputs<E, TIER, MODE>(s, key0, cnt, wp, s_stt, st, so);
 }
 
-// Two-pass emission (MODE_EMIT) from a CONVERGED warp -- the staged scan's
-// per-byte and per-chunk loops only (a full-mask vote in the divergent
-// callers, halo warm-ups and re-walks, would deadlock).  f = this lane
-// reaches output state x at key0.  A single-output state's record is stored
-// by its own lane; the records of a multi-output state are written by the
-// whole warp, one such lane at a time: 32 consecutive ids read and 32
-// consecutive records written per instruction.  Per-lane loops cost one
-// L1 wavefront per record for the id and another for the store (each lane
-// writes its own chain's range: 32 lines per instruction), which is what
-// bound dense dictionaries (C5 English: 4-14 outputs per flagged byte).
+// Two-pass emission (MODE_EMIT) from a CONVERGED warp -- used by the SPLIT
+// re-walk only (a full-mask vote in the divergent callers, halo warm-ups and
+// re-walks, would deadlock).  f = this lane reaches output state x at key0.
+// States with fewer than AC_COOP_MIN outputs are written by their own lane;
+// the records of larger output sets are written by the whole warp,
+// AC_COOP_BATCH such states at a time: 32 consecutive ids read and 32
+// consecutive records written per instruction, where a per-lane loop costs
+// one L1 wavefront per record for the id and another for the store (each
+// lane writes its own chain's range: 32 lines per instruction).  Measured
+// (C5 English, 256 MiB, list): SPLIT 20K patterns (13.5 outputs per flagged
+// byte) 11.8 -> 8.2 ms; in the GLOBAL tier's per-byte loop (English 5K,
+// 4.3 outputs per flagged byte, 64-register kernel) every form was slower
+// than the per-lane branch -- 4.30 ms vs 4.7 (all multi-output states
+// cooperative), 5.0-5.4 (thresholds 6-12), 5.6-16 (batches of 2-8 states:
+// register pressure) -- so that loop keeps emit_outputs.
 #ifndef AC_COOP_MIN
-#define AC_COOP_MIN 2  // smallest |output(x)| written by the whole warp
+#define AC_COOP_MIN 8  // smallest |output(x)| written by the whole warp
 #endif
 #ifndef AC_COOP_BATCH
-#define AC_COOP_BATCH 1  // multi-output states whose id loads are in flight together
+#define AC_COOP_BATCH 2  // multi-output states whose id loads are in flight together
 #endif
 #ifndef AC_COOP
-#define AC_COOP 1  // 0: per-lane emission in the two-pass MODE_EMIT loops (ablation)
+#define AC_COOP 1  // 0: per-lane emission in the SPLIT two-pass re-walk (ablation)
 #endif
 template <typename E, int TIER>
 __device__ __forceinline__ void emit_coop(uint32_t x, uint32_t f, uint64_t key0, uint64_t &wp, const E *s_stt,
@@ -1141,22 +1148,6 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                         else
                             emit_loop(std::false_type{});
                         cnt[0] = (uint32_t)(-nk);
-                    } else if constexpr (MODE == MODE_EMIT && AC_COOP) {
-                        // two-pass emission (dense outputs): one flagged byte
-                        // per lane per round, multi-output states written by
-                        // the whole warp (emit_coop)
-                        while (__any_sync(0xffffffffu, fm)) {
-                            const uint32_t act = fm != 0;
-                            const int bb = act ? 31 - __clz(fm) : 0;
-                            fm &= ~(act << bb);
-                            const int i = bb >> 1;
-                            const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
-                            const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
-                            const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
-                            const uint32_t pr = (i & 4) ? b1 : b0;
-                            const uint32_t x = (bb & 1) ? (pr & 0xFFFFu) : (pr >> 16);
-                            emit_coop<E, TIER>(x, act, kb[0] + ((uint64_t)bb << 24), wp[0], s_stt, st, so);
-                        }
                     } else
                     while (__any_sync(0xffffffffu, fm)) {
                         if (fm) {
@@ -1241,19 +1232,6 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                             if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k])
                                 emit_outputs<E, TIER, MODE>(s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
                                                             st, so);
-                        }
-                    }
-                } else if constexpr (MODE == MODE_EMIT && AC_COOP) {
-                    // two-pass emission (dense outputs), warp-cooperative
-#pragma unroll
-                    for (int bb = 15; bb >= 0; --bb) {
-#pragma unroll
-                        for (int k = 0; k < K; k++) {
-                            const uint32_t e = next_entry<E, TIER>(s_stt, st, s[k],
-                                                                   class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
-                            s[k] = state_of<E, TIER>(e, st);
-                            const uint32_t f = flag_of<E, TIER>(e, s[k], st) & (live[k] ? 1u : 0u);
-                            emit_coop<E, TIER>(s[k], f, kb[k] + ((uint64_t)bb << 24), wp[k], s_stt, st, so);
                         }
                     }
                 } else {

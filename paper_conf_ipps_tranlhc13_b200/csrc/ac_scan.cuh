@@ -136,8 +136,7 @@ struct StagedConfig {
     X(8, 32, 1, 32, 2, 0)     \
     X(9, 16, 2, 16, 2, 1)     \
     X(10, 32, 1, 32, 1, 1)    \
-    X(11, 32, 1, 32, 1, 0)    \
-    X(12, 16, 2, 32, 1, 1)
+    X(11, 32, 1, 32, 1, 0)
 
 // Kernel entry points (host side launchers); all return cudaError_t.
 cudaError_t launch_scan_global(int mode, uint32_t entry_bytes, uint32_t tier, const uint8_t *text,
