@@ -219,6 +219,16 @@ __device__ __forceinline__ uint32_t class_of(const uint8_t *s_cmap, uint32_t byt
     }
 }
 
+// The same with the identity known at compile time (the SPLIT auto variant
+// is also instantiated for identity class maps, e.g. C3: no predicated load).
+template <int TIER, bool IDENT>
+__device__ __forceinline__ uint32_t class_of_k(const uint8_t *s_cmap, uint32_t byte, const SttView &st) {
+    if constexpr (IDENT)
+        return byte;
+    else
+        return class_of<TIER>(s_cmap, byte, st);
+}
+
 // Entry -> next state and output flag.
 template <typename E, int TIER>
 __device__ __forceinline__ uint32_t state_of(uint32_t e, const SttView &st) {
@@ -878,7 +888,8 @@ struct StagedShape {
     static_assert(SLOT % 512 == 0 || W == 16, "slots must keep the swizzle atom aligned");
 };
 
-template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1>
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1,
+          bool IDENT = false>
 __global__ void __launch_bounds__(WARPS * 32, 1)
     k_scan_staged(const __grid_constant__ CUtensorMap tmap, const uint8_t *__restrict__ mtext, SttView st,
                   StagedGeom g, ScanOut so) {
@@ -1187,7 +1198,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
                         for (int bb = 15; bb >= 0; --bb) {
                             const uint32_t e =
-                                next_entry<E, TIER>(s_stt, st, s[k], class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                                next_entry<E, TIER>(s_stt, st, s[k], class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                             s[k] = state_of<E, TIER>(e, st);
                             fm |= flag_of<E, TIER>(e, s[k], st) << bb;
                         }
@@ -1201,7 +1212,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll 1
                                 for (int bb = 15; bb >= 0; --bb) {
                                     const uint32_t e = next_entry<E, TIER>(
-                                        s_stt, st, x, class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                                        s_stt, st, x, class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                                     x = state_of<E, TIER>(e, st);
                                     emit_coop<E, TIER>(x, (fm >> bb) & 1u, kb[k] + ((uint64_t)bb << 24), wp[k], s_stt,
                                                        st, so);
@@ -1212,7 +1223,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll 1
                             for (int bb = 15; bb >= 0; --bb) {
                                 const uint32_t e = next_entry<E, TIER>(
-                                    s_stt, st, x, class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                                    s_stt, st, x, class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                                 x = state_of<E, TIER>(e, st);
                                 if ((fm >> bb) & 1u)
                                     emit_outputs<E, TIER, MODE>(x, kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
@@ -1227,7 +1238,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
                         for (int k = 0; k < K; k++) {
                             const uint32_t e =
-                                next_entry<E, TIER>(s_stt, st, s[k], class_of<TIER>(s_cmap, byte_of(v[k], bb), st));
+                                next_entry<E, TIER>(s_stt, st, s[k], class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                             s[k] = state_of<E, TIER>(e, st);
                             if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k])
                                 emit_outputs<E, TIER, MODE>(s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
@@ -1390,10 +1401,11 @@ cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_tota
     }
 }
 
-template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1>
+template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1,
+          bool IDENT = false>
 static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
                                    const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
-    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE, STRIDE>;
+    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE, STRIDE, IDENT>;
     const StagedConfig cfg{WARPS, K, W, NST, SWIZZLE};
     const size_t smem = staged_smem_bytes(cfg, smem_stt);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1416,6 +1428,12 @@ static cudaError_t launch_staged_m(int variant, const CUtensorMap &tmap, const u
             if (variant == 7) return launch_staged_v<E, TIER, MODE, 32, 1, 16, 2, 1, 2>(tmap, mtext, st, g, so, smem_stt, s);
         }
         return cudaErrorInvalidValue;
+    }
+    if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT)) {
+        // the SPLIT auto variant (10) for identity class maps: no class-map
+        // load in the walk (list modes; ptxas spills the count-mode forms)
+        if (variant == 10 && st.cmap_ident)
+            return launch_staged_v<E, TIER, MODE, 32, 1, 32, 1, 1, 1, true>(tmap, mtext, st, g, so, smem_stt, s);
     }
     switch (variant) {
 #define AC_CASE(i, w, k, wd, ns, sw) \
