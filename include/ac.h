@@ -153,13 +153,16 @@ typedef struct {
     uint64_t stt2_bytes;
     /* SPLIT tier (valid when split_bytes != 0): split_dense + 1 dense rows of
      * split_dstride u16 entries (row r = BFS state r for r < split_dense, the
-     * last one all 0xFFFF), then one 8-byte record per sparse hot state
-     * split_dense <= s < split_records: {lo32 = fd | c1 << 16 | c2 << 24,
-     * hi32 = t1 | t2 << 16}, delta(s, c) = t1 if c == c1, t2 if c == c2, else
-     * row[fd][c]; dense states read row[s][c]; a u16 entry is 2 x + flag, or
-     * 0xFFFF = read the global table; split_cold_records sparse states point
-     * at the 0xFFFF row; states >= split_records are read from the global
-     * table. */
+     * last one -- the escape row -- all 0xFFFF), then one 8-byte CHILDREN
+     * record per hot state split_dense <= s < split_records:
+     * {lo32 = c1 | c2 << 8 | c3 << 16 | c4 << 24 (the classes of s's goto
+     * children, ascending, the last one repeated),
+     * hi32 = fd | flags << 12 | (2 first - 1) << 16}: delta(s, c) = first + k
+     * (flag bit k) for the lowest k with c == c_k, else row[fd][c] (fd = f(s),
+     * dense); dense states read row[s][c]; a u16 result is 2 x + flag, and a
+     * value > 0xFFFD means "read the global table".  split_cold_records
+     * records are cold (fd = the escape row, 2 first - 1 = 0xFFFD); states
+     * >= split_records are read from the global table. */
     uint32_t split_dense, split_records, split_dstride, split_cold_records;
     uint64_t split_bytes;
 } ac_stt_info;

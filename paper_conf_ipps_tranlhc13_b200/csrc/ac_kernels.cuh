@@ -167,18 +167,18 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
 __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
     const uint32_t rep = cls * 0x01010101u;
     const uint32_t sparse = (s - st.s_dense) < (st.s_rec - st.s_dense);
-    const uint32_t rbase = base + st.s_rec_x0;  // loop-invariant: one uniform register
-    uint32_t lo = rbase + s * 8u;               // record address (biased by -8 s_dense)
+    uint32_t lo = base + st.s_rec_x0 + s * 8u;  // record address (biased by -8 s_dense)
     uint32_t hi = min(s, st.s_dense);           // fd of a dense state (itself) or of a cold one (escape row)
     asm("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.v2.u32 {%0, %1}, [%0];\n\t"
         "@!p xor.b32 %0, %3, 0x80808080;\n\t}"
         : "+r"(lo), "+r"(hi)
         : "r"(sparse), "r"(rep));
-    // lo = c1 | c2 << 8 | c3 << 16 | c4 << 24, hi = fd | first << 12 | flags << 27
+    // lo = c1 | c2 << 8 | c3 << 16 | c4 << 24, hi = fd | flags << 12 | (2 first - 1) << 16
     const uint32_t x = lo ^ rep;                                  // a zero byte where a class matches
     const uint32_t z = (x - 0x01010101u) & ~x & 0x80808080u;      // lowest set bit: the first match
-    const uint32_t kk = (__ffs(z) - 1u) >> 3;                      // child index (garbage if no match)
-    const uint32_t child = ((((hi >> 12) & 0x7FFFu) + kk) << 1) | ((hi >> (27u + kk)) & 1u);
+    const uint32_t p = __ffs(z) - 1u;                              // 8 k + 7 (garbage if no match)
+    // 2 (first + k) = (2 first - 1) + (p >> 2), then child k's output flag
+    const uint32_t child = ((hi >> 16) + (p >> 2)) | ((hi >> (12u + (p >> 3))) & 1u);
     // e16 = child if a class matched, else the shared row entry row[fd][cls]:
     // one predicate for the load and the select
     uint32_t e16 = base + (hi & 0xFFFu) * st.s_row_bytes + cls * 2u;

@@ -18,14 +18,17 @@
 //     (the levels whose states mostly have more than four children);
 //   * the next level [D, H) gets an 8-byte CHILDREN record per state:
 //       lo = c1 | c2 << 8 | c3 << 16 | c4 << 24   (children's classes, ascending)
-//       hi = fd | first << 12 | flags << 27
+//       hi = fd | flags << 12 | (2 first - 1) << 16
 //     delta(s, c) = first + k if c == c_k (k = 0..3: BFS numbers a state's
 //     children consecutively in class order), else row[fd][c] -- fd = f(s),
 //     which is dense, so the exceptions of s against fd are exactly its
 //     goto children; flags bit k = output(first + k) != {}.  Fewer than four
 //     children repeat the last class; a state with more (or ids that do not
-//     fit) is COLD: fd = D (the ESCAPE row, all 0xFFFF) and first = 0x7FFF,
-//     so any result escapes;
+//     fit) is COLD: fd = D (the ESCAPE row, all 0xFFFF) and 2 first - 1 =
+//     0xFFFD, so any result escapes.  (first is stored doubled minus one: the
+//     scan adds the match position p = 8 k + 7 as p >> 2 = 2 k + 1 and gets
+//     2 (first + k) -- the 16-bit entry form -- in one instruction; first >= 1
+//     because a child is never the root);
 //   * states >= H are COLD.
 // A 16-bit result is 2 x + flag (x = BFS id, flag = output(x) != {}) for
 // x < 32767, and > 0xFFFD means "read the 32-bit dense table in global
@@ -122,24 +125,35 @@ bool split_table(ac_table &t, size_t budget) {
         for (uint32_t i = 0; ok && i < k; i++) ok = (tgt[i] & 0x7fffffffu) == (tgt[0] & 0x7fffffffu) + i;
         ok = ok && (k == 0 || (tgt[0] & 0x7fffffffu) + k - 1 < 32767u);
         uint32_t lo, hi;
+        const uint32_t kCold = D | (0xFFFDu << 16);  // cold: every result escapes
         if (!ok) {
             lo = 0;
-            hi = D | (0x7FFFu << 12);  // cold: every result escapes
+            hi = kCold;
             n_cold++;
         } else if (k == 0) {
-            // a leaf: every class falls back to row[fd]; the record's class
-            // bytes (all 0) hit class 0, so "child" 0 is delta(s, 0) itself
-            const uint32_t e0 = delta(s, 0);
-            lo = 0;
-            hi = (e0 & 0x7fffffffu) < 32767u ? fd[s] | ((e0 & 0x7fffffffu) << 12) | ((e0 >> 31) << 27)
-                                             : D | (0x7FFFu << 12);
-            n_cold += (e0 & 0x7fffffffu) >= 32767u;
+            // a leaf: every class falls back to row[fd]; the record names one
+            // class c* (all four bytes) whose "child" is delta(s, c*) itself
+            // -- a class whose target is not the root (first >= 1)
+            uint32_t cs = C;
+            for (uint32_t c = 0; c < C && cs == C; c++) {
+                const uint32_t x = delta(s, c) & 0x7fffffffu;
+                if (x >= 1 && x < 32767u) cs = c;
+            }
+            if (cs == C) {
+                lo = 0;
+                hi = kCold;
+                n_cold++;
+            } else {
+                const uint32_t e = delta(s, cs);
+                lo = cs * 0x01010101u;
+                hi = fd[s] | ((e >> 31) << 12) | ((2 * (e & 0x7fffffffu) - 1) << 16);
+            }
         } else {
             for (uint32_t i = k; i < 4; i++) cls[i] = cls[k - 1];  // repeats never win (lowest byte first)
             uint32_t flags = 0;
             for (uint32_t i = 0; i < k; i++) flags |= (tgt[i] >> 31) << i;
             lo = cls[0] | (cls[1] << 8) | (cls[2] << 16) | (cls[3] << 24);
-            hi = fd[s] | ((tgt[0] & 0x7fffffffu) << 12) | (flags << 27);
+            hi = fd[s] | (flags << 12) | ((2 * (tgt[0] & 0x7fffffffu) - 1) << 16);
         }
         std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8], &lo, 4);
         std::memcpy(&blob[dense_bytes + (size_t)(s - D) * 8 + 4], &hi, 4);

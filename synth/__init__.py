@@ -228,7 +228,7 @@ def patterns_kmers(text: np.ndarray, count: int, seed: int, lmin: int = 20, lmax
 # ---------------------------------------------------------------------------
 def text_repeat(n: int, unit: bytes) -> np.ndarray:
     u = np.frombuffer(unit, dtype=np.uint8)
-    return np.resize(u, n).astype(np.uint8)
+    return np.resize(u, n)  # uint8, one n-byte allocation (C5 texts reach 16 GiB)
 
 
 def patterns_runs(byte: int, kmax: int) -> list[bytes]:

@@ -287,19 +287,19 @@ def _decode_split(t):
     rec = blob[(D + 1) * ds * 2:].view(np.uint32).reshape(-1, 2).astype(np.int64)
     cls4 = np.stack([(rec[:, 0] >> (8 * i)) & 0xFF for i in range(4)], axis=1)      # children's classes
     fd = rec[:, 1] & 0xFFF
-    first = (rec[:, 1] >> 12) & 0x7FFF
-    flags = rec[:, 1] >> 27
-    assert (fd <= D).all()
+    flags = (rec[:, 1] >> 12) & 0xF
+    f2 = rec[:, 1] >> 16  # 2 first - 1
+    assert (fd <= D).all() and (f2 % 2 == 1).all()
     c = np.arange(C)[None, :]
-    # first matching class byte k (lowest index) -> child first + k
+    # first matching class byte k (lowest index) -> child first + k (16-bit form 2 x + flag)
     k = np.full((H - D, C), -1, np.int64)
     for i in range(3, -1, -1):
         k = np.where(cls4[:, i:i + 1] == c, i, k)
-    child = ((first[:, None] + np.maximum(k, 0)) << 1) | ((flags[:, None] >> np.maximum(k, 0)) & 1)
+    child = (f2[:, None] + 1 + 2 * np.maximum(k, 0)) | ((flags[:, None] >> np.maximum(k, 0)) & 1)
     e16_sparse = np.where(k >= 0, child, rows[fd])
     e16 = np.concatenate([rows[:D], e16_sparse])
     E = (e16 >> 1) | ((e16 & 1) << 31)
-    cold = (fd == D) & (first == 0x7FFF)
+    cold = (fd == D) & (f2 == 0xFFFD)
     return np.where(e16 > 0xFFFD, -1, E), int(cold.sum())
 
 
