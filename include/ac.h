@@ -189,16 +189,22 @@ typedef struct {
                               scratch slot during the single emitting pass
                               (0 = auto from cap); chains with more are
                               re-scanned straight into place                 */
-    uint32_t two_pass;     /* list mode: 0 = auto: single emitting pass, or
-                              the two passes when cap > n (room for more
-                              than one record per text byte); single pass: chain
+    uint32_t two_pass;     /* list mode: 0 = auto: single emitting pass;
+                              when cap > n (room for more than one record
+                              per text byte: dense outputs) the EVENTS
+                              single pass if the table has 32-bit entries
+                              and < 2^24 states (one parked event per output
+                              state reached, expanded into records by the
+                              gather), else the two passes; single pass: chain
                               offsets computed inside the staged scan when
                               the text pointer is 16-byte aligned, else by
                               a separate offset scan); 1 = count pass + emit
                               pass (ablation / fallback); 2 = single pass
                               with the separate offset scan (ablation);
                               3 = single pass with 8-byte scratch records
-                              (ablation of the 4-byte narrow records)      */
+                              (ablation of the 4-byte narrow records);
+                              4 = the EVENTS single pass whenever the table
+                              allows it (else as 0)                         */
     uint32_t stride;       /* 0 = the table's default, 1 = force one byte
                               per lookup even if a two-byte table exists     */
     uint32_t n_events;     /* pairs available in `events`                    */

@@ -510,13 +510,28 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     // caller's density bound: room for more than one record per owned text
     // byte selects the two-pass emission (no count pass is needed to plan).
     const bool dense_out = (!opts || (opts->two_pass == 0 && opts->scratch_slots == 0)) && cap > n_owned;
-    bool two_pass = (opts && opts->two_pass == 1) || dense_out;
-    // single pass: each chain keeps its first q records in a scratch slot;
-    // if the slots cannot be allocated the call falls back to two passes
+    // EVENTS (dense outputs): a single emitting pass that parks one event per
+    // output state reached (an event per flagged byte, not a record per
+    // match), so a slot of chain-length entries never overflows; k_gather
+    // expands the events into records with coalesced, full-sector writes.
+    // Needs the 32-bit table (its rows carry the output summary k_gather
+    // reads) and state ids below 2^24 (an event is start << 24 | state).
+    // Measured (C5 English, 256 MiB, list): see DESIGN.md section 7.
+    const uint64_t max_len = std::max<uint64_t>(g.n_chains ? g.chain_len : 0,
+                                                std::max(ra.n_chains ? ra.chain_len : 0, rb.n_chains ? rb.chain_len : 0));
+    const uint64_t max_ev_scratch = 32ull << 30;
+    const bool ev_ok = eb == 4 && h->host.n_states < (1u << 24) && max_len > 0 &&
+                       n_chains * max_len * 8 <= max_ev_scratch;
+    bool events = ev_ok && ((opts && opts->two_pass == 4) || dense_out);
+    bool two_pass = (opts && opts->two_pass == 1) || (dense_out && !events);
+    // single pass: each chain keeps its first q records (or all its events)
+    // in a scratch slot; if the slots cannot be allocated the call falls back
+    // to two passes
     uint64_t q = opts && opts->scratch_slots ? opts->scratch_slots : 4 * (cap / n_chains) + 64;
     if (q > kMaxSlots) q = kMaxSlots;
     const uint64_t max_scratch = 8ull << 30;
     if (n_chains * q * 8 > max_scratch) q = max_scratch / (n_chains * 8);
+    if (events) q = max_len;
     if (q == 0) q = 1;
     void *scratch = nullptr;
     if (!two_pass) {
@@ -525,6 +540,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             cudaGetLastError();
             scratch = nullptr;
             two_pass = true;
+            events = false;
         }
     }
     // in-kernel offsets: the staged kernel places its chains (decoupled
@@ -535,7 +551,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     const uint64_t R = (uint64_t)cfg.warps * 32 * cfg.k;
     const uint64_t n_lb = place ? (g.n_chains + R - 1) / R : 0;  // staged CTAs
     const size_t tiles = offsets_tiles(n_chains);
-    const size_t bytes = n_chains * 8 * 3 + tiles * 8 + 16 + n_lb * 8;
+    const size_t bytes = n_chains * 8 * 3 + tiles * 8 + 16 + n_lb * 8 + (events ? n_chains * 4 : 0);
     void *ws = nullptr;
     {
         cudaError_t e = ws_alloc(&ws, bytes, stream, h->device);
@@ -551,6 +567,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     unsigned int *counter = reinterpret_cast<unsigned int *>(tile_state + tiles);
     unsigned int *list_n = counter + 1;
     unsigned long long *lb = place ? reinterpret_cast<unsigned long long *>(counter + 4) : nullptr;
+    uint32_t *chain_events = events ? reinterpret_cast<uint32_t *>(counter + 4 + 2 * n_lb) : nullptr;
+    so.chain_events = chain_events;
     so.tile_state = lb;
     so.ticket = place ? counter + 2 : nullptr;
     so.chain_end_w = chain_end;
@@ -567,6 +585,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     }
     nm_bits = nm.nbits;
     g_scratch_rec = two_pass ? 0u : nm.nbits ? 4u : 8u;
+    const EventExpand evx{chain_events, static_cast<const uint32_t *>(h->d_stt), h->host.row_stride, h->host.info_col,
+                         h->d_out_ids};
     so.chain_counts = counts;
     so.chain_end = chain_end;
     if (scratch) {
@@ -593,7 +613,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
             post("k_offsets", stream, 0);
         }
         pre(stream);
-        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, tp, nm,
+        AC_CUDA(launch_gather(counts, chain_end, n_chains, so.scratch, so.q, so.out, d_res, list, list_n, tp, nm, evx,
                               h->num_sms, stream),
                 "k_gather");
         post("k_gather", stream, 0);

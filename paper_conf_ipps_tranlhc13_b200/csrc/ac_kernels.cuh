@@ -391,6 +391,14 @@ __device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t
             for (uint32_t j = p + c; j > p; --j) so.out[--wp] = key0 | __ldg(st.out_ids + j - 1);
         }
     } else if constexpr (MODE == MODE_EMIT_OPT) {
+        if (so.chain_events) {
+            // EVENTS (dense outputs): one entry per output state reached, the
+            // slot pointer moves down (a slot holds a whole chain's events)
+            *reinterpret_cast<uint64_t *>(wp) = key0 | x;
+            wp -= 8;
+            cnt += c;
+            return;
+        }
         uint64_t *last = reinterpret_cast<uint64_t *>(wp);
         const uint32_t p = out_payload<E, TIER>(s_stt, st, x);
         if (c == 1) {
@@ -648,6 +656,10 @@ __global__ void __launch_bounds__(GT) k_scan_global(const uint8_t *__restrict__ 
         walk_global<E, TIER, MODE, false>(text, own_hi, walk_hi, s, cnt, wp, s_cmap, s_stt, st, so);
         walk_global<E, TIER, MODE, true>(text, lo, own_hi, s, cnt, wp, s_cmap, s_stt, st, so);
         if constexpr (MODE == MODE_COUNT_CHAINS || MODE == MODE_EMIT_OPT) so.chain_counts[g] = cnt;
+        if constexpr (MODE == MODE_EMIT_OPT)
+            if (so.chain_events)
+                so.chain_events[g] =
+                    (uint32_t)((reinterpret_cast<uint64_t>(so.scratch + (g + 1) * so.q - 1) - wp) >> 3);
     }
     if constexpr (MODE == MODE_COUNT_TOTAL) {
         const unsigned long long tot = warp_sum((unsigned long long)cnt);
@@ -1276,6 +1288,17 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
         for (int k = 0; k < K; k++)
             if (live[k]) so.chain_counts[g.chain0 + row0 + k * 32 + lane] = cnt[k];
+    }
+    if constexpr (MODE == MODE_EMIT_OPT) {
+        if (so.chain_events) {
+#pragma unroll
+            for (int k = 0; k < K; k++) {
+                const uint64_t c = g.chain0 + row0 + k * 32 + lane;
+                if (live[k])
+                    so.chain_events[c] = (uint32_t)((reinterpret_cast<uint64_t>(so.scratch + (c + 1) * so.q - 1) -
+                                                     wp[k]) >> 3);
+            }
+        }
     }
     if constexpr (MODE == MODE_EMIT_OPT) {
         if (place) place_chains<K>(so, g, wring, ring, Sh::WARP_RING, WARPS, tile, row0, cnt, live);

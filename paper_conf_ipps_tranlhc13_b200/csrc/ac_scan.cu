@@ -135,7 +135,7 @@ static constexpr uint64_t kMaxTail = 256;
 __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ counts, uint64_t *chain_end,
                                                 uint64_t n_chains, const uint64_t *__restrict__ scratch, uint32_t q,
                                                 uint64_t *__restrict__ out, ac_result *res, uint64_t *list,
-                                                unsigned int *list_n, TailPlace tp, NarrowMain nm) {
+                                                unsigned int *list_n, TailPlace tp, NarrowMain nm, EventExpand ev) {
     const int lane = threadIdx.x & 31;
     uint64_t main_total = 0;
     if (tp.tile_state) {
@@ -173,6 +173,57 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
             if (lane == 0) chain_end[c] = end;  // k_rewalk reads it for listed chains
         }
         if (cnt == 0) continue;
+        if (ev.events) {
+            // EVENTS: the chain's events, canonical order, at the slot's end;
+            // 32 at a time: each lane reads its event's output summary, a warp
+            // scan places the records, and the warp writes them 32 consecutive
+            // records per round (full 32-byte sectors) -- each record's owner
+            // is the last event starting at or before it
+            const uint32_t ne = ev.events[c];
+            if (ne > q) {
+                if (lane == 0) list[atomicAdd(list_n, 1u)] = c;
+                continue;
+            }
+            const uint64_t *src = scratch + c * q + (q - ne);
+            uint64_t run = end - cnt;  // index of the chain's first record
+            uint32_t le;
+            asm("mov.u32 %0, %%lanemask_le;" : "=r"(le));
+            for (uint32_t i0 = 0; i0 < ne; i0 += 32) {
+                const bool has = i0 + lane < ne;
+                const uint64_t e = has ? __ldg(src + i0 + lane) : 0ull;
+                uint32_t p = 0, cx = 0;
+                if (has) {
+                    const uint32_t *row = ev.stt + (uint64_t)(e & 0xFFFFFFu) * ev.stride + ev.info_col;
+                    p = __ldg(row);
+                    cx = __ldg(row + 1);
+                }
+                uint32_t incl = cx;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += t;
+                }
+                const uint32_t excl = incl - cx, T = __shfl_sync(0xffffffffu, incl, 31);
+                const uint32_t khi = (uint32_t)(e >> 32), klo = (uint32_t)e & 0xFF000000u;
+                for (uint32_t R = 0; R < T; R += 32) {
+                    // record positions in (R, R + 32) where an event's records start
+                    const uint32_t starts =
+                        __reduce_or_sync(0xffffffffu, (cx && excl > R && excl < R + 32) ? 1u << (excl - R) : 0u);
+                    const int o0 = __popc(__ballot_sync(0xffffffffu, cx && excl <= R)) - 1;  // owner of record R
+                    const int own = o0 + __popc(starts & le);
+                    const uint32_t po = __shfl_sync(0xffffffffu, p, own), co = __shfl_sync(0xffffffffu, cx, own);
+                    const uint32_t eo = __shfl_sync(0xffffffffu, excl, own);
+                    const uint32_t kh = __shfl_sync(0xffffffffu, khi, own), kl = __shfl_sync(0xffffffffu, klo, own);
+                    const uint32_t r = R + lane;
+                    if (r < T) {
+                        const uint32_t id = co == 1u ? po : __ldg(ev.out_ids + po + (r - eo));
+                        out[run + r] = ((uint64_t)kh << 32) | kl | id;
+                    }
+                }
+                run += T;
+            }
+            continue;
+        }
         if (cnt > q) {
             if (lane == 0) list[atomicAdd(list_n, 1u)] = c;
             continue;
@@ -211,12 +262,12 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
 cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t n_chains,
                           const uint64_t *scratch, uint32_t q, uint64_t *out, ac_result *res,
                           uint64_t *list, unsigned int *list_n, const TailPlace &tp, const NarrowMain &nm,
-                          int num_sms, cudaStream_t stream) {
+                          const EventExpand &ev, int num_sms, cudaStream_t stream) {
     if (n_chains == 0) return cudaSuccess;
     if (tp.tile_state && tp.tail_n > kMaxTail) return cudaErrorInvalidValue;
     const uint64_t want = (n_chains + 7) / 8;
     const unsigned grid = (unsigned)(want < (uint64_t)num_sms * 8 ? want : (uint64_t)num_sms * 8);
-    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp, nm);
+    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp, nm, ev);
     return cudaGetLastError();
 }
 

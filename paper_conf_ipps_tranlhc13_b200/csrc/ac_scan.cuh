@@ -83,6 +83,22 @@ struct ScanOut {
     // running CTA is itself running or done -- CUDA does not promise that
     // CTAs start in blockIdx order
     unsigned int *ticket;
+    // MODE_EMIT_OPT EVENTS (dense outputs, 32-bit tables, S < 2^24; NULL =
+    // off): the scan parks one 8-byte event (start << 24 | state) per output
+    // state reached instead of its records -- the slot holds a whole chain's
+    // events (q >= chain length) -- counts the records for the offsets as
+    // usual and writes the chain's event count here; k_gather expands the
+    // events into records, warp-cooperatively and coalesced
+    uint32_t *chain_events;
+};
+
+// What k_gather needs to expand events: the 32-bit table's output summary
+// (payload at info_col, count at info_col + 1 of each row) and the CSR ids.
+struct EventExpand {
+    const uint32_t *events;   // per-chain event counts (NULL = record mode)
+    const uint32_t *stt;
+    uint32_t stride, info_col;
+    const uint32_t *out_ids;
 };
 
 // Decoupled look-back words: 2-bit flag (aggregate / inclusive prefix) + value.
@@ -157,7 +173,7 @@ size_t staged_smem_bytes(const StagedConfig &cfg, size_t smem_stt_bytes);
 cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t n_chains,
                           const uint64_t *scratch, uint32_t q, uint64_t *out, ac_result *res,
                           uint64_t *list, unsigned int *list_n, const TailPlace &tp, const NarrowMain &nm,
-                          int num_sms, cudaStream_t stream);
+                          const EventExpand &ev, int num_sms, cudaStream_t stream);
 cudaError_t launch_rewalk(uint32_t entry_bytes, uint32_t tier, const uint8_t *text, uint64_t n_total,
                           const SttView &st, const Region &a, const Region &b, const StagedGeom &g,
                           const ScanOut &so, const uint64_t *list, const unsigned int *list_n, size_t smem_stt,

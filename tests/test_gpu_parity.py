@@ -49,7 +49,9 @@ def gpu_keys(stt, text_np: np.ndarray, **kw) -> np.ndarray:
         _, r3 = ac.match(stt, t, scratch_slots=2, **kw)  # most chains overflow -> k_rewalk
         _, r4 = ac.match(stt, t, two_pass=2, **kw)  # single pass with the separate offset scan
         _, r5 = ac.match(stt, t, two_pass=3, **kw)  # single pass with wide scratch records
+        _, r6 = ac.match(stt, t, two_pass=4, **kw)  # EVENTS single pass (32-bit tables; else as auto)
         assert torch.equal(r2, recs) and torch.equal(r3, recs) and torch.equal(r4, recs) and torch.equal(r5, recs)
+        assert torch.equal(r6, recs)
     assert cnt == c
     return recs.cpu().numpy()
 
