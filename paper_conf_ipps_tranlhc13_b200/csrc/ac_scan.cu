@@ -132,7 +132,10 @@ size_t offsets_tiles(uint64_t n) { return (size_t)((n + OTILE - 1) / OTILE); }
 // writes the count and the capacity status.
 static constexpr uint64_t kMaxTail = 256;
 
-__global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ counts, uint64_t *chain_end,
+// EV: the chains hold events (EVENTS single pass), else records; the record
+// copy keeps 32 registers (8 CTAs of 256 threads per SM: one wave)
+template <bool EV>
+__global__ void __launch_bounds__(256, EV ? 1 : 8) k_gather(const uint64_t *__restrict__ counts, uint64_t *chain_end,
                                                 uint64_t n_chains, const uint64_t *__restrict__ scratch, uint32_t q,
                                                 uint64_t *__restrict__ out, ac_result *res, uint64_t *list,
                                                 unsigned int *list_n, TailPlace tp, NarrowMain nm, EventExpand ev) {
@@ -173,7 +176,7 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
             if (lane == 0) chain_end[c] = end;  // k_rewalk reads it for listed chains
         }
         if (cnt == 0) continue;
-        if (ev.events) {
+        if constexpr (EV) {
             // EVENTS: the chain's events, canonical order, at the slot's end;
             // 32 at a time: each lane reads its event's output summary, a warp
             // scan places the records, and the warp writes them 32 consecutive
@@ -188,15 +191,24 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
             uint64_t run = end - cnt;  // index of the chain's first record
             uint32_t le;
             asm("mov.u32 %0, %%lanemask_le;" : "=r"(le));
-            for (uint32_t i0 = 0; i0 < ne; i0 += 32) {
-                const bool has = i0 + lane < ne;
-                const uint64_t e = has ? __ldg(src + i0 + lane) : 0ull;
-                uint32_t p = 0, cx = 0;
-                if (has) {
+            // one chunk of 32 events: the event and its output summary
+            auto fetch = [&](uint32_t i0, uint64_t &e, uint32_t &p, uint32_t &cx) {
+                e = 0;
+                p = cx = 0;
+                if (i0 + lane < ne) {
+                    e = __ldg(src + i0 + lane);
                     const uint32_t *row = ev.stt + (uint64_t)(e & 0xFFFFFFu) * ev.stride + ev.info_col;
                     p = __ldg(row);
                     cx = __ldg(row + 1);
                 }
+            };
+            uint64_t e_n;
+            uint32_t p_n, cx_n;
+            fetch(0, e_n, p_n, cx_n);
+            for (uint32_t i0 = 0; i0 < ne; i0 += 32) {
+                const uint64_t e = e_n;
+                const uint32_t p = p_n, cx = cx_n;
+                if (i0 + 32 < ne) fetch(i0 + 32, e_n, p_n, cx_n);  // the next chunk's loads in flight
                 uint32_t incl = cx;
 #pragma unroll
                 for (int o = 1; o < 32; o <<= 1) {
@@ -205,19 +217,31 @@ __global__ void __launch_bounds__(256) k_gather(const uint64_t *__restrict__ cou
                 }
                 const uint32_t excl = incl - cx, T = __shfl_sync(0xffffffffu, incl, 31);
                 const uint32_t khi = (uint32_t)(e >> 32), klo = (uint32_t)e & 0xFF000000u;
-                for (uint32_t R = 0; R < T; R += 32) {
-                    // record positions in (R, R + 32) where an event's records start
-                    const uint32_t starts =
-                        __reduce_or_sync(0xffffffffu, (cx && excl > R && excl < R + 32) ? 1u << (excl - R) : 0u);
-                    const int o0 = __popc(__ballot_sync(0xffffffffu, cx && excl <= R)) - 1;  // owner of record R
-                    const int own = o0 + __popc(starts & le);
-                    const uint32_t po = __shfl_sync(0xffffffffu, p, own), co = __shfl_sync(0xffffffffu, cx, own);
-                    const uint32_t eo = __shfl_sync(0xffffffffu, excl, own);
-                    const uint32_t kh = __shfl_sync(0xffffffffu, khi, own), kl = __shfl_sync(0xffffffffu, klo, own);
-                    const uint32_t r = R + lane;
-                    if (r < T) {
-                        const uint32_t id = co == 1u ? po : __ldg(ev.out_ids + po + (r - eo));
-                        out[run + r] = ((uint64_t)kh << 32) | kl | id;
+                // rounds of 32 records, four at a time: every id load of the
+                // batch is issued before its stores
+                constexpr int RB = 4;
+                for (uint32_t R0 = 0; R0 < T; R0 += 32 * RB) {
+                    uint32_t id[RB], kh[RB], kl[RB];
+#pragma unroll
+                    for (int u = 0; u < RB; u++) {
+                        const uint32_t R = R0 + 32u * u;
+                        // record positions in (R, R + 32) where an event's records start
+                        const uint32_t starts = __reduce_or_sync(
+                            0xffffffffu, (cx && excl > R && excl < R + 32) ? 1u << (excl - R) : 0u);
+                        const int o0 = __popc(__ballot_sync(0xffffffffu, cx && excl <= R)) - 1;  // owner of R
+                        const int own = o0 + __popc(starts & le);
+                        const uint32_t po = __shfl_sync(0xffffffffu, p, own), co = __shfl_sync(0xffffffffu, cx, own);
+                        const uint32_t eo = __shfl_sync(0xffffffffu, excl, own);
+                        kh[u] = __shfl_sync(0xffffffffu, khi, own);
+                        kl[u] = __shfl_sync(0xffffffffu, klo, own);
+                        const uint32_t r = R + lane;
+                        id[u] = po;
+                        if (r < T && co != 1u) id[u] = __ldg(ev.out_ids + po + (r - eo));
+                    }
+#pragma unroll
+                    for (int u = 0; u < RB; u++) {
+                        const uint32_t r = R0 + 32u * u + lane;
+                        if (r < T) out[run + r] = ((uint64_t)kh[u] << 32) | kl[u] | id[u];
                     }
                 }
                 run += T;
@@ -267,7 +291,12 @@ cudaError_t launch_gather(const uint64_t *counts, uint64_t *chain_end, uint64_t 
     if (tp.tile_state && tp.tail_n > kMaxTail) return cudaErrorInvalidValue;
     const uint64_t want = (n_chains + 7) / 8;
     const unsigned grid = (unsigned)(want < (uint64_t)num_sms * 8 ? want : (uint64_t)num_sms * 8);
-    k_gather<<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp, nm, ev);
+    if (ev.events)
+        k_gather<true><<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp, nm,
+                                                 ev);
+    else
+        k_gather<false><<<grid, 256, 0, stream>>>(counts, chain_end, n_chains, scratch, q, out, res, list, list_n, tp,
+                                                  nm, ev);
     return cudaGetLastError();
 }
 

@@ -41,6 +41,7 @@ def main():
     p.add_argument("--list", action="store_true")
     p.add_argument("--exact-cap", action="store_true", help="list buffer of exactly count records")
     p.add_argument("--policies", default="0", help="text L2 policies (0 auto, 1 evict-normal, 2 evict-first)")
+    p.add_argument("--two-pass", default="0", help="ac_match_opts.two_pass values to time (0 auto, 1 two passes, 4 events)")
     a = p.parse_args()
     for name in a.workloads.split(","):
         w = synth.make(name, n=a.n)
@@ -55,10 +56,11 @@ def main():
                 continue
             cap = ac.count(stt, text) if a.exact_cap else n // 8 + 64
             out = torch.empty(max(1, cap), dtype=torch.int64, device="cuda") if a.list else None
-            for v, pol in [(v, pol) for v in a.variants.split(",") for pol in a.policies.split(",")]:
+            for v, pol, tpm in [(v, pol, tpm) for v in a.variants.split(",") for pol in a.policies.split(",")
+                                for tpm in a.two_pass.split(",")]:
                 tpol, prom, win = (pol + ":0:0").split(":")[:3]  # text policy[:promotion[:L2 window MiB]]
                 knobs = dict(kernel=ac.KERNEL_STAGED, variant=int(v), text_policy=int(tpol), text_promotion=int(prom),
-                             l2_window_mib=int(win))
+                             l2_window_mib=int(win), two_pass=int(tpm))
                 try:
                     ac.match_async(stt, text, out, res, **knobs)
                 except ac.AcError as e:
@@ -66,7 +68,8 @@ def main():
                     continue
                 t = timeit(lambda: ac.match_async(stt, text, out, res, **knobs))
                 print(json.dumps({"workload": name, "n": n, "tier": stt.tier_name, "variant": int(v),
-                                  "policy": pol, "list": bool(a.list), "exact_cap": bool(a.exact_cap),
+                                  "policy": pol, "two_pass": int(tpm), "list": bool(a.list),
+                                  "exact_cap": bool(a.exact_cap),
                                   "states": stt.info["n_states"], "split_dense": stt.info["split_dense"],
                                   "split_records": stt.info["split_records"], "ms": round(t, 4),
                                   "gbps": round(n * 8 / t / 1e6, 1), "matches": int(res[0]),
