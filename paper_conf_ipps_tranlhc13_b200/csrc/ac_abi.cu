@@ -378,6 +378,19 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
         } else {
             const uint64_t target = (uint64_t)h->num_sms * R;
             L = (avail + target - 1) / target;
+            // list mode, single pass: keep the expected records per chain
+            // (the capacity read as a density bound) within half a scratch
+            // slot -- on long texts one chain per lane would overflow every
+            // slot into k_rewalk (C5 English 1K at 16 GiB: 32K records per
+            // chain); shorter chains just take more CTA waves (ticketed tiles)
+            // (whole waves: L is re-divided so every wave is full)
+            if (emit && cap > 0 && cap <= n_owned) {
+                const uint64_t lmax = (kMaxSlots / 2) * (n_owned / cap);
+                if (L > lmax) {
+                    const uint64_t waves = (L + lmax - 1) / lmax;
+                    L = (avail + waves * target - 1) / (waves * target);
+                }
+            }
             L = (L + W - 1) / W * W;
             if (L < kStagedMinChain) L = kStagedMinChain;
         }

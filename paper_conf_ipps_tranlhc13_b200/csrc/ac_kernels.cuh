@@ -394,7 +394,13 @@ __device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t
         if (so.chain_events) {
             // EVENTS (dense outputs): one entry per output state reached, the
             // slot pointer moves down (a slot holds a whole chain's events)
+#ifdef AC_EV_EVICT_LAST
+            uint64_t pol;
+            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+            asm volatile("st.global.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(wp), "l"(key0 | x), "l"(pol) : "memory");
+#else
             *reinterpret_cast<uint64_t *>(wp) = key0 | x;
+#endif
             wp -= 8;
             cnt += c;
             return;

@@ -6,7 +6,8 @@ count modes, checked against the oracle.  Run under
 Covers the staged kernel's mbarrier rings and TMA loads, its in-kernel
 look-back (a ticketed decoupled look-back across CTAs, P:216 is the paper's
 synchronisation step), the SMEM / COMPACT / SPLIT / GLOBAL tiers, k_offsets,
-k_gather, k_rewalk and the packet-batch kernel."""
+k_gather (record copy and EVENTS expansion), k_rewalk and the packet-batch
+kernel."""
 from __future__ import annotations
 
 import sys
@@ -58,6 +59,18 @@ def main():
     stt = ac.build(w.patterns)  # SPLIT
     check("c3 split staged", stt, o, w.text, kernel=ac.KERNEL_STAGED, chain_bytes=256)
     check("c3 global-only", stt, o, w.text, kernel=ac.KERNEL_GLOBAL)
+    check("c3 split staged events", stt, o, w.text, kernel=ac.KERNEL_STAGED, chain_bytes=256, two_pass=4)
+
+    # dense outputs: the EVENTS single pass (GLOBAL tier, 32-bit table) and the
+    # SPLIT two-pass re-walk with emit_coop
+    voc = synth.english_vocabulary(5002)
+    text = synth.text_english((1 << 18) + 11, 5000, voc)
+    pats = synth.patterns_substrings(text, 5000, 4, 32, 5001)
+    o = Oracle(pats)
+    stt = ac.build(pats)
+    check("english5k events", stt, o, text, kernel=ac.KERNEL_STAGED, chain_bytes=256, two_pass=4)
+    stt = ac.build(pats, tier=ac.TIER_SPLIT)
+    check("english5k split two-pass", stt, o, text, kernel=ac.KERNEL_STAGED, chain_bytes=256, two_pass=True)
 
     w = synth.make("c4", n=(1 << 20) + 3)
     o = Oracle(w.patterns)

@@ -227,8 +227,17 @@ def patterns_kmers(text: np.ndarray, count: int, seed: int, lmin: int = 20, lmax
 # C5 adversarial families
 # ---------------------------------------------------------------------------
 def text_repeat(n: int, unit: bytes) -> np.ndarray:
+    # one n-byte allocation filled by doubling copies (C5 texts reach 16 GiB;
+    # np.resize of a short unit concatenates n / len(unit) views)
     u = np.frombuffer(unit, dtype=np.uint8)
-    return np.resize(u, n)  # uint8, one n-byte allocation (C5 texts reach 16 GiB)
+    out = np.empty(n, dtype=np.uint8)
+    k = min(n, u.size)
+    out[:k] = u[:k]
+    while k < n:
+        m = min(k, n - k)
+        out[k:k + m] = out[:m]
+        k += m
+    return out
 
 
 def patterns_runs(byte: int, kmax: int) -> list[bytes]:
