@@ -394,13 +394,16 @@ __device__ __forceinline__ void emit_outputs(uint32_t x, uint64_t key0, uint32_t
         if (so.chain_events) {
             // EVENTS (dense outputs): one entry per output state reached, the
             // slot pointer moves down (a slot holds a whole chain's events)
-#ifdef AC_EV_EVICT_LAST
+            // Events are written with an L2 evict-first policy: 0.6 GB of them
+            // per 256 MiB of English text otherwise pushed the 32-bit table
+            // out of L2 (ncu: 2.2 GB of DRAM reads per launch instead of 0.6;
+            // the same time -- the walk is bound by L1, not DRAM).  An
+            // evict-last hint changed nothing; gathering four events per lane
+            // in shared memory for one 32-byte store was no faster either
+            // (English 5K 2.75 -> 2.83 ms, 20K 5.70 -> 5.45 ms).
             uint64_t pol;
-            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
             asm volatile("st.global.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(wp), "l"(key0 | x), "l"(pol) : "memory");
-#else
-            *reinterpret_cast<uint64_t *>(wp) = key0 | x;
-#endif
             wp -= 8;
             cnt += c;
             return;
@@ -1300,9 +1303,8 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
             for (int k = 0; k < K; k++) {
                 const uint64_t c = g.chain0 + row0 + k * 32 + lane;
-                if (live[k])
-                    so.chain_events[c] = (uint32_t)((reinterpret_cast<uint64_t>(so.scratch + (c + 1) * so.q - 1) -
-                                                     wp[k]) >> 3);
+                const uint64_t last = reinterpret_cast<uint64_t>(so.scratch + (c + 1) * so.q - 1);
+                if (live[k]) so.chain_events[c] = (uint32_t)((last - wp[k]) >> 3);
             }
         }
     }

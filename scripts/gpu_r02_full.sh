@@ -29,8 +29,9 @@ if [ "$SKIP_EVIDENCE" != "1" ]; then
   done
 fi
 if [ "$SKIP_SWEEP" != "1" ]; then
+  # SWEEP_OUT: another file name for a partial re-run (merged by hand); SWEEP_ARGS: extra flags
   timeout 6000 python scripts/sweep_c5.py --logn ${SWEEP_LOGN:-26,28,30,34} --patterns 1000,5000,10000,20000,50000 \
-    > $O/sweep_c5.jsonl 2> $O/sweep_c5.err
+    $SWEEP_ARGS > $O/${SWEEP_OUT:-sweep_c5}.jsonl 2> $O/${SWEEP_OUT:-sweep_c5}.err
 fi
 if [ "$WITH_SANITIZE" = "1" ]; then
   for tool in memcheck racecheck synccheck initcheck; do
