@@ -212,7 +212,7 @@ def _check_text(text: torch.Tensor):
 
 
 def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, scratch_slots: int = 0,
-           two_pass: bool = False, events=None, stride: int = 0, text_policy: int = 0, text_promotion: int = 0,
+           two_pass: int = 0, events=None, stride: int = 0, text_policy: int = 0, text_promotion: int = 0,
            l2_window_mib: int = 0):
     o = ac_match_opts(ctypes.sizeof(ac_match_opts), kernel, chain_bytes, variant, scratch_slots,
                       int(two_pass), stride, 0, None, text_policy, text_promotion, l2_window_mib)
@@ -226,11 +226,12 @@ def _mopts(kernel: int = KERNEL_AUTO, chain_bytes: int = 0, variant: int = 0, sc
 
 def match_async(stt: Stt, text: torch.Tensor, out: torch.Tensor | None, result: torch.Tensor, *,
                 n_halo: int = 0, base: int = 0, stream=None, kernel: int = KERNEL_AUTO, chain_bytes: int = 0,
-                variant: int = 0, scratch_slots: int = 0, two_pass: bool = False, stride: int = 0,
+                variant: int = 0, scratch_slots: int = 0, two_pass: int = 0, stride: int = 0,
                 events=None, text_policy: int = 0, text_promotion: int = 0, l2_window_mib: int = 0) -> int:
     """Enqueue the scan; result (int64[2] CUDA) receives (count, status).
     ``text`` holds n_owned + n_halo bytes.  ``kernel``/``chain_bytes``/
-    ``variant``/``scratch_slots``/``two_pass`` select the scan (ac_match_opts).  ``events``: optional list
+    ``variant``/``scratch_slots``/``two_pass`` select the scan (ac_match_opts; ``two_pass``: 0 auto,
+    1 two passes, 2/3 single-pass ablations, 4 the EVENTS single pass).  ``events``: optional list
     of (start, end) torch.cuda.Event pairs (already created, i.e. recorded
     once) recorded around each kernel launch.  Returns the number of kernel
     launches issued."""
