@@ -544,6 +544,12 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     if (q > kMaxSlots) q = kMaxSlots;
     const uint64_t max_scratch = 8ull << 30;
     if (n_chains * q * 8 > max_scratch) q = max_scratch / (n_chains * 8);
+    // a scratch budget too small for twice the expected records per chain
+    // would send most chains to k_rewalk (C5 English 1K at 16 GiB, 4.8 G
+    // records: 380 slots for ~1.7 K records per chain): two passes instead
+    if (!events && !two_pass && (!opts || (opts->two_pass == 0 && opts->scratch_slots == 0)) &&
+        q < 2 * (cap / n_chains))
+        two_pass = true;
     if (events) q = max_len;
     if (q == 0) q = 1;
     void *scratch = nullptr;

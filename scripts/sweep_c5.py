@@ -151,7 +151,7 @@ def main():
         K = len(w.patterns)
         point("c5-adv-a-28", w.patterns, w.text, closed_form=K * n - K * (K - 1) // 2)
         w = synth.make("c5-adv-p-28")
-        point("c5-adv-p-28", w.patterns, w.text, list_budget=4 << 30)
+        point("c5-adv-p-28", w.patterns, w.text)
 
 
 if __name__ == "__main__":
