@@ -527,13 +527,14 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     // output state reached (an event per flagged byte, not a record per
     // match), so a slot of chain-length entries never overflows; k_gather
     // expands the events into records with coalesced, full-sector writes.
-    // Needs the 32-bit table (its rows carry the output summary k_gather
-    // reads) and state ids below 2^24 (an event is start << 24 | state).
+    // Needs a dense table whose rows carry the output summary k_gather reads
+    // (every tier but COMPACT, whose states are renumbered) and state ids
+    // below 2^24 (an event is start << 24 | state).
     // Measured (C5 English, 256 MiB, list): see DESIGN.md section 7.
     const uint64_t max_len = std::max<uint64_t>(g.n_chains ? g.chain_len : 0,
                                                 std::max(ra.n_chains ? ra.chain_len : 0, rb.n_chains ? rb.chain_len : 0));
     const uint64_t max_ev_scratch = 32ull << 30;
-    const bool ev_ok = eb == 4 && h->host.n_states < (1u << 24) && max_len > 0 &&
+    const bool ev_ok = (eb == 4 || h->tier != AC_TIER_COMPACT) && h->host.n_states < (1u << 24) && max_len > 0 &&
                        n_chains * max_len * 8 <= max_ev_scratch;
     bool events = ev_ok && ((opts && opts->two_pass == 4) || dense_out);
     bool two_pass = (opts && opts->two_pass == 1) || (dense_out && !events);
@@ -596,7 +597,7 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     // chain per lane, 16-bit table, one byte per lookup): offset in chain and
     // pattern id must share 32 bits.  Off for the two-pass ablation.
     NarrowMain nm{0, g.chain0, g.n_chains, base + g.m0, g.chain_len};
-    if (!two_pass && g.n_chains && cfg.k == 1 && eb == 2 && !ss.stt2 && !(opts && opts->two_pass == 3)) {
+    if (!two_pass && !events && g.n_chains && cfg.k == 1 && eb == 2 && !ss.stt2 && !(opts && opts->two_pass == 3)) {
         uint32_t pid_bits = 1, off_bits = 1;
         while ((1ull << pid_bits) < h->host.n_patterns) pid_bits++;
         while ((1ull << off_bits) < g.chain_len) off_bits++;
@@ -604,8 +605,8 @@ static ac_status match_async(const ac_stt *h, const uint8_t *d_text, uint64_t n_
     }
     nm_bits = nm.nbits;
     g_scratch_rec = two_pass ? 0u : nm.nbits ? 4u : 8u;
-    const EventExpand evx{chain_events, static_cast<const uint32_t *>(h->d_stt), h->host.row_stride, h->host.info_col,
-                         h->d_out_ids};
+    const EventExpand evx{chain_events, h->d_stt,       h->host.row_stride, h->host.info_col,
+                          eb,           h->d_out_off, h->d_out_ids};
     so.chain_counts = counts;
     so.chain_end = chain_end;
     if (scratch) {

@@ -1175,7 +1175,41 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                                 nk -= (int32_t)c;
                             }
                         };
-                        if (nb)
+                        bool done = false;
+                        if constexpr (TIER != AC_TIER_COMPACT) {
+                            if (so.chain_events) {
+                                // EVENTS (dense outputs): one event per flagged byte
+                                // (start << 24 | state), the slot pointer moves down;
+                                // only the output count is read here
+                                uint64_t pol;
+                                asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+                                for (uint32_t it = 0; it < iters; ++it) {
+                                    uint32_t bb;
+                                    asm("bfind.u32 %0, %1;" : "=r"(bb) : "r"(fm));
+                                    const uint32_t act = fm != 0;
+                                    fm &= ~(1u << (bb & 31u));
+                                    const uint32_t i = bb >> 1;
+                                    const uint32_t a0 = (i & 1) ? hist[1] : hist[0], a1 = (i & 1) ? hist[3] : hist[2];
+                                    const uint32_t a2 = (i & 1) ? hist[5] : hist[4], a3 = (i & 1) ? hist[7] : hist[6];
+                                    const uint32_t b0 = (i & 2) ? a1 : a0, b1 = (i & 2) ? a3 : a2;
+                                    const uint32_t pr = (i & 4) ? b1 : b0;
+                                    const uint32_t x = __byte_perm(pr, 0, (bb & 1) ? 0x4410 : 0x4432);
+                                    uint32_t c = out_info_pred<E, TIER, false>(s_stt, st, x, act).y;
+                                    if (sizeof(E) == 2 && c == 0xFFFFu)
+                                        c = __ldg(st.out_off + x + 1) - __ldg(st.out_off + x);
+                                    asm volatile(
+                                        "{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %3, 0;\n\t"
+                                        "@p st.global.L2::cache_hint.u64 [%0], %1, %2;\n\t}" ::"l"(wp[0]),
+                                        "l"((kb[0] + ((uint64_t)(bb & 15u) << 24)) | x), "l"(pol), "r"(act)
+                                        : "memory");
+                                    wp[0] -= (uint64_t)act << 3;
+                                    nk -= (int32_t)c;
+                                }
+                                done = true;
+                            }
+                        }
+                        if (done) {
+                        } else if (nb)
                             emit_loop(std::true_type{});
                         else
                             emit_loop(std::false_type{});

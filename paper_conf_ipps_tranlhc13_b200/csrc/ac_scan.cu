@@ -197,9 +197,17 @@ __global__ void __launch_bounds__(256, EV ? 1 : 8) k_gather(const uint64_t *__re
                 p = cx = 0;
                 if (i0 + lane < ne) {
                     e = __ldg(src + i0 + lane);
-                    const uint32_t *row = ev.stt + (uint64_t)(e & 0xFFFFFFu) * ev.stride + ev.info_col;
-                    p = __ldg(row);
-                    cx = __ldg(row + 1);
+                    const uint32_t x = (uint32_t)e & 0xFFFFFFu;
+                    if (ev.entry_bytes == 4) {
+                        const uint32_t *row = static_cast<const uint32_t *>(ev.stt) + (uint64_t)x * ev.stride + ev.info_col;
+                        p = __ldg(row);
+                        cx = __ldg(row + 1);
+                    } else {
+                        const uint16_t *row = static_cast<const uint16_t *>(ev.stt) + (uint64_t)x * ev.stride + ev.info_col;
+                        p = __ldg(reinterpret_cast<const uint32_t *>(row));
+                        cx = __ldg(row + 2);
+                        if (cx == 0xFFFFu) cx = __ldg(ev.out_off + x + 1) - __ldg(ev.out_off + x);
+                    }
                 }
             };
             uint64_t e_n;

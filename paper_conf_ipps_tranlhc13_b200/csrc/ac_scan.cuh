@@ -92,13 +92,15 @@ struct ScanOut {
     uint32_t *chain_events;
 };
 
-// What k_gather needs to expand events: the 32-bit table's output summary
-// (payload at info_col, count at info_col + 1 of each row) and the CSR ids.
+// What k_gather needs to expand events: the dense table's per-row output
+// summary (32-bit entries: payload at entry info_col, count at info_col + 1;
+// 16-bit entries: u32 payload at entries [info_col, info_col + 1], u16 count
+// at info_col + 2, 0xFFFF = read the CSR offsets) and the CSR.
 struct EventExpand {
     const uint32_t *events;   // per-chain event counts (NULL = record mode)
-    const uint32_t *stt;
-    uint32_t stride, info_col;
-    const uint32_t *out_ids;
+    const void *stt;
+    uint32_t stride, info_col, entry_bytes;
+    const uint32_t *out_off, *out_ids;
 };
 
 // Decoupled look-back words: 2-bit flag (aggregate / inclusive prefix) + value.
