@@ -192,10 +192,12 @@ typedef struct {
     uint32_t two_pass;     /* list mode: 0 = auto: single emitting pass;
                               when cap > n (room for more than one record
                               per text byte: dense outputs) the EVENTS
-                              single pass if the table has 32-bit entries
-                              and < 2^24 states (one parked event per output
-                              state reached, expanded into records by the
-                              gather), else the two passes; single pass: chain
+                              single pass unless the STT is COMPACT (one
+                              parked event per output state reached,
+                              expanded into records by the gather), else the
+                              two passes -- also chosen when the scratch
+                              budget cannot hold twice the expected records
+                              per chain; single pass: chain
                               offsets computed inside the staged scan when
                               the text pointer is 16-byte aligned, else by
                               a separate offset scan); 1 = count pass + emit
