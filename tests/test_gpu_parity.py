@@ -144,6 +144,24 @@ def test_dense_outputs_english(P, tier):
     assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED), want)
 
 
+@pytest.mark.parametrize("tier", [ac.TIER_SMEM, ac.TIER_GLOBAL])
+def test_saturated_output_counts(tier):
+    """70,000 copies of one pattern (reading R5: every id reported): |output|
+    exceeds the 16-bit row count (0xFFFF -> CSR offsets) and one event expands
+    into more records than a gather chunk's rounds hold; every emission mode
+    (gpu_keys: auto, two passes, overflow re-walk, EVENTS) against the oracle."""
+    pats = [b"ab"] * 70000 + [b"b", b"zab"]
+    rng = np.random.default_rng(5)
+    text = rng.choice(np.frombuffer(b"abz", np.uint8), size=(1 << 12) + 3)
+    o = Oracle(pats)
+    stt = ac.build(pats, tier=tier)
+    assert stt.info["entry_bytes"] == 2 and stt.info["tier"] == tier
+    want = oracle_keys(o, text)
+    assert want.size > 70000 * 100
+    assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED), want)
+    assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_GLOBAL), want)
+
+
 def test_compact_is_auto_for_c2():
     w = synth.make("c2", n=1 << 20)
     stt = ac.build(w.patterns)
