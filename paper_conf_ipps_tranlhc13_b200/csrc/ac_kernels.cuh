@@ -164,6 +164,10 @@ __device__ __forceinline__ uint32_t compact_next(uint32_t base, const SttView &s
 // (the class bytes of a non-record lane are cls ^ 0x80, which never match).
 // A 16-bit result above 0xFFFD -- cold state, cold record or a next id >=
 // 32767 -- is replaced by the full entry from the global table (L1/L2).
+// IDENT: identity class map, so C = 256 and the 32-bit table's row stride is
+// the compile-time (256 + 2) | 1 = 259 (one constant-bank load less per step).
+static constexpr uint32_t kIdentStride = 259;
+template <bool IDENT = false>
 __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st, uint32_t s, uint32_t cls) {
     const uint32_t rep = cls * 0x01010101u;
     const uint32_t sparse = (s - st.s_dense) < (st.s_rec - st.s_dense);
@@ -196,7 +200,7 @@ __device__ __forceinline__ uint32_t split_next(uint32_t base, const SttView &st,
         // load doubled the long-scoreboard stalls, C3 list 3.2 -> 5.4 ms/GiB;
         // an L2 evict-last hint on this load: no change.)
         // (S x row_stride < 2^32 entries, checked by ac_build: a 32-bit index)
-        const uint32_t *gp = static_cast<const uint32_t *>(st.stt) + (s * st.stride + cls);
+        const uint32_t *gp = static_cast<const uint32_t *>(st.stt) + (s * (IDENT ? kIdentStride : st.stride) + cls);
         asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(g) : "l"(gp));
     }
     return g;
@@ -245,12 +249,12 @@ __device__ __forceinline__ uint32_t flag_of(uint32_t e, uint32_t x, const SttVie
         return e >> (8 * sizeof(E) - 1);
 }
 
-template <typename E, int TIER>
+template <typename E, int TIER, bool IDENT = false>
 __device__ __forceinline__ uint32_t next_entry(const E *s_stt, const SttView &st, uint32_t s, uint32_t cls) {
     if constexpr (TIER == AC_TIER_COMPACT) {
         return compact_next(smem_u32(s_stt), st, s, cls);
     } else if constexpr (TIER == AC_TIER_SPLIT) {
-        return split_next(smem_u32(s_stt), st, s, cls);
+        return split_next<IDENT>(smem_u32(s_stt), st, s, cls);
     } else {
         return stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, s * st.stride + cls);
     }
@@ -1253,7 +1257,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
                         for (int bb = 15; bb >= 0; --bb) {
                             const uint32_t e =
-                                next_entry<E, TIER>(s_stt, st, s[k], class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
+                                next_entry<E, TIER, IDENT>(s_stt, st, s[k], class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                             s[k] = state_of<E, TIER>(e, st);
                             fm |= flag_of<E, TIER>(e, s[k], st) << bb;
                         }
@@ -1266,7 +1270,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                                 uint32_t x = s_in;
 #pragma unroll 1
                                 for (int bb = 15; bb >= 0; --bb) {
-                                    const uint32_t e = next_entry<E, TIER>(
+                                    const uint32_t e = next_entry<E, TIER, IDENT>(
                                         s_stt, st, x, class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                                     x = state_of<E, TIER>(e, st);
                                     emit_coop<E, TIER>(x, (fm >> bb) & 1u, kb[k] + ((uint64_t)bb << 24), wp[k], s_stt,
@@ -1277,7 +1281,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                             uint32_t x = s_in;
 #pragma unroll 1
                             for (int bb = 15; bb >= 0; --bb) {
-                                const uint32_t e = next_entry<E, TIER>(
+                                const uint32_t e = next_entry<E, TIER, IDENT>(
                                     s_stt, st, x, class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                                 x = state_of<E, TIER>(e, st);
                                 if ((fm >> bb) & 1u)
@@ -1293,7 +1297,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
 #pragma unroll
                         for (int k = 0; k < K; k++) {
                             const uint32_t e =
-                                next_entry<E, TIER>(s_stt, st, s[k], class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
+                                next_entry<E, TIER, IDENT>(s_stt, st, s[k], class_of_k<TIER, IDENT>(s_cmap, byte_of(v[k], bb), st));
                             s[k] = state_of<E, TIER>(e, st);
                             if (__builtin_expect(flag_of<E, TIER>(e, s[k], st) != 0, 0) && live[k])
                                 emit_outputs<E, TIER, MODE>(s[k], kb[k] + ((uint64_t)bb << 24), cnt[k], wp[k], s_stt,
@@ -1497,7 +1501,7 @@ static cudaError_t launch_staged_m(int variant, const CUtensorMap &tmap, const u
     if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT)) {
         // the SPLIT auto variant (10) for identity class maps: no class-map
         // load in the walk (list modes; ptxas spills the count-mode forms)
-        if (variant == 10 && st.cmap_ident)
+        if (variant == 10 && st.cmap_ident && st.stride == kIdentStride)
             return launch_staged_v<E, TIER, MODE, 32, 1, 32, 1, 1, 1, true>(tmap, mtext, st, g, so, smem_stt, s);
     }
     switch (variant) {
