@@ -411,12 +411,19 @@ def test_capacity_error_and_count_only():
     assert c == need
 
 
-def test_shard_api_concatenation():
-    w = synth.make("c2", n=(3 << 20) + 11, n_patterns=400)
-    o = Oracle(w.patterns)
-    want = oracle_keys(o, w.text)
-    stt = ac.build(w.patterns)
-    t = torch.from_numpy(w.text).cuda()
+@pytest.mark.parametrize("which", ["c2", "english5k-events"])
+def test_shard_api_concatenation(which):
+    if which == "c2":
+        w = synth.make("c2", n=(3 << 20) + 11, n_patterns=400)
+        text, pats, kw = w.text, w.patterns, {}
+    else:  # dense outputs: shards through the EVENTS single pass (base offsets in the events)
+        voc = synth.english_vocabulary(5002)
+        text = synth.text_english((1 << 20) + 11, 5000, voc)
+        pats, kw = synth.patterns_substrings(text, 5000, 4, 32, 5001), {"two_pass": 4}
+    o = Oracle(pats)
+    want = oracle_keys(o, text)
+    stt = ac.build(pats)
+    t = torch.from_numpy(text).cuda()
     n = t.numel()
     rng = np.random.default_rng(1)
     for G in (2, 3, 8):
@@ -425,7 +432,7 @@ def test_shard_api_concatenation():
         parts = []
         for lo, hi in zip(bounds[:-1], bounds[1:]):
             halo = min(stt.maxlen - 1, n - hi)
-            c, recs = ac.match(stt, t[lo:hi + halo], n_halo=halo, base=lo)
+            c, recs = ac.match(stt, t[lo:hi + halo], n_halo=halo, base=lo, **kw)
             parts.append(recs.cpu().numpy())
         assert_same(np.concatenate(parts), want)
 
