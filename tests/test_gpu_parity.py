@@ -142,6 +142,14 @@ def test_dense_outputs_english(P, tier):
     want = oracle_keys(o, text)
     assert want.size > text.size // 5
     assert_same(gpu_keys(stt, text, kernel=ac.KERNEL_STAGED), want)
+    # one record short: the capacity status and the needed count, nothing written
+    t = torch.from_numpy(text).cuda()
+    out = torch.full((want.size - 1,), -1, dtype=torch.int64, device="cuda")
+    for tp in (0, 1, 4):
+        with pytest.raises(ac.CapacityError) as ei:
+            ac.match(stt, t, out, two_pass=tp)
+        assert ei.value.count == want.size
+    assert bool((out == -1).all())
 
 
 @pytest.mark.parametrize("tier", [ac.TIER_SMEM, ac.TIER_GLOBAL])
