@@ -217,6 +217,7 @@ static SttView view_of(const ac_stt *h, int v) {
     s.stride2 = h->host.stride2;
     s.n_classes = h->host.n_classes;
     s.sblob = nullptr;
+    s.cnt8 = 0;
     s.s_dense = s.s_rec = s.s_row_bytes = s.s_rec_x0 = 0;
     s.cmap_ident = 1;
     for (int b = 0; b < 256; b++) s.cmap_ident &= h->host.class_map[b] == b ? 1u : 0u;
@@ -245,6 +246,12 @@ static SttView view_of(const ac_stt *h, int v) {
     const uint64_t cap = stt_budget(h, v) / row_bytes(h);
     s.smem_rows = (uint32_t)(rows < cap ? rows : cap);
     s.smem_bytes = (uint32_t)(s.smem_rows * row_bytes(h));
+    if (h->tier == AC_TIER_GLOBAL && h->d_cnt8 && v && h->host.n_states <= stt_budget(h, v)) {
+        // the staged kernel keeps every state's output count in shared memory
+        s.sblob = h->d_cnt8;
+        s.smem_bytes = h->host.n_states;
+        s.cnt8 = 1;
+    }
     return s;
 }
 
@@ -265,6 +272,8 @@ static void free_device(ac_stt *h) {
     h->d_stt2 = nullptr;
     cudaFree(h->d_split);
     h->d_split = nullptr;
+    cudaFree(h->d_cnt8);
+    h->d_cnt8 = nullptr;
     cudaFree(h->d_class_map);
     cudaFree(h->d_out_off);
     cudaFree(h->d_out_ids);
@@ -1163,6 +1172,15 @@ ac_status ac_build(const uint8_t *const *patterns, const uint32_t *lens, uint32_
             return fail(e, "cudaMemset(split)");
         if ((e = cudaMemcpy(h->d_split, t.split.data(), t.split.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
             return fail(e, "H2D split");
+    }
+    if (tier == AC_TIER_GLOBAL && t.entry_bytes == 4) {
+        // per-state output counts for the staged GLOBAL scan (view_of)
+        std::vector<uint8_t> c8((t.n_states + 15) / 16 * 16, 0);
+        for (uint32_t x = 0; x < t.n_states; x++)
+            c8[x] = (uint8_t)std::min<uint32_t>(t.out_off[x + 1] - t.out_off[x], 255u);
+        if ((e = cudaMalloc(&h->d_cnt8, c8.size())) != cudaSuccess) return fail(e, "cudaMalloc(cnt8)");
+        if ((e = cudaMemcpy(h->d_cnt8, c8.data(), c8.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
+            return fail(e, "H2D cnt8");
     }
     const std::vector<uint8_t> &blob = tier == AC_TIER_COMPACT ? t.compact : t.stt;
     const size_t stt_alloc = (blob.size() + 15) / 16 * 16 + 16;

@@ -60,6 +60,7 @@ struct ac_stt {
     uint32_t *d_stt2 = nullptr;      // two-byte table (NEXT-4) or NULL
     void *d_split = nullptr;         // SPLIT tier: the shared-memory part (dense rows + records)
     uint8_t *d_class_map = nullptr;  // 256 B
+    uint8_t *d_cnt8 = nullptr;       // GLOBAL tier, 32-bit table: min(|output(s)|, 255) per state (staged)
     uint32_t *d_out_off = nullptr;
     uint32_t *d_out_ids = nullptr;
     uint32_t *d_lens = nullptr;

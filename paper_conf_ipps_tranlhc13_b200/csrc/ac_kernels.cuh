@@ -282,6 +282,12 @@ __device__ __forceinline__ uint32_t out_count(const E *s_stt, const SttView &st,
     if constexpr (TIER == AC_TIER_COMPACT) {
         return compact_out<E>(s_stt, st, s).y;
     } else {
+        if constexpr (TIER == AC_TIER_GLOBAL) {
+            if (st.cnt8) {  // staged counts (GLOBAL tier, staged kernel)
+                const uint32_t c8 = reinterpret_cast<const uint8_t *>(s_stt)[s];
+                if (c8 != 255u) return c8;
+            }
+        }
         const uint32_t idx = s * st.stride + st.info_col + (sizeof(E) == 2 ? 2 : 1);
         uint32_t c = stt_load<E, TIER>(s_stt, static_cast<const E *>(st.stt), st.smem_rows, s, idx);
         if (sizeof(E) == 2 && c == 0xFFFFu) c = __ldg(st.out_off + s + 1) - __ldg(st.out_off + s);

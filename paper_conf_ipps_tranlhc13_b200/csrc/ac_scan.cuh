@@ -48,6 +48,10 @@ struct SttView {
     const void *sblob;
     uint32_t s_dense, s_rec, s_row_bytes, s_rec_x0;
     uint32_t cmap_ident;  // the class map is the identity (every byte occurs in a pattern)
+    // GLOBAL tier, staged kernel: `sblob` holds min(|output(s)|, 255) per state,
+    // staged into shared memory -- a flagged lane reads its output count there
+    // instead of from the table row in L1/L2 (255 = read the row)
+    uint32_t cnt8;
 };
 
 // A run of equal-length chains over owned starts [lo, hi) of the shard.
