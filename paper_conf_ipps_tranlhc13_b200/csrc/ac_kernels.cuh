@@ -919,8 +919,10 @@ struct StagedShape {
     static_assert(SLOT % 512 == 0 || W == 16, "slots must keep the swizzle atom aligned");
 };
 
+// DENSE (SPLIT, EVENTS): emit inline at each flagged byte instead of the
+// flag walk + re-walk, which for dense dictionaries walks most chunks twice
 template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1,
-          bool IDENT = false>
+          bool IDENT = false, bool DENSE = false>
 __global__ void __launch_bounds__(WARPS * 32, 1)
     k_scan_staged(const __grid_constant__ CUtensorMap tmap, const uint8_t *__restrict__ mtext, SttView st,
                   StagedGeom g, ScanOut so) {
@@ -1249,7 +1251,7 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                                                     live[k], s_cmap, s_stt, st, so);
                     }
                 } else if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT) &&
-                                     !kSplitInlineEmit) {
+                                     !kSplitInlineEmit && !DENSE) {
                     // rare matches (the tier is chosen for large byte
                     // dictionaries): the 16 steps only collect the flag bits
                     // -- the count-mode loop, no record keys or slot
@@ -1297,7 +1299,8 @@ __global__ void __launch_bounds__(WARPS * 32, 1)
                         }
                     }
                 } else if constexpr (TIER == AC_TIER_SPLIT) {
-                    // counting with rare matches: the walk is the whole loop
+                    // counting with rare matches, or emitting inline (DENSE):
+                    // the walk is the whole loop
 #pragma unroll
                     for (int bb = 15; bb >= 0; --bb) {
 #pragma unroll
@@ -1477,10 +1480,10 @@ cudaError_t launch_rewalk_tier(uint32_t eb, const uint8_t *text, uint64_t n_tota
 }
 
 template <typename E, int TIER, int MODE, int WARPS, int K, int W, int NST, int SWIZZLE, int STRIDE = 1,
-          bool IDENT = false>
+          bool IDENT = false, bool DENSE = false>
 static cudaError_t launch_staged_v(const CUtensorMap &tmap, const uint8_t *mtext, const SttView &st,
                                    const StagedGeom &g, const ScanOut &so, size_t smem_stt, cudaStream_t stream) {
-    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE, STRIDE, IDENT>;
+    auto kern = k_scan_staged<E, TIER, MODE, WARPS, K, W, NST, SWIZZLE, STRIDE, IDENT, DENSE>;
     const StagedConfig cfg{WARPS, K, W, NST, SWIZZLE};
     const size_t smem = staged_smem_bytes(cfg, smem_stt);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1507,6 +1510,12 @@ static cudaError_t launch_staged_m(int variant, const CUtensorMap &tmap, const u
     if constexpr (TIER == AC_TIER_SPLIT && (MODE == MODE_EMIT || MODE == MODE_EMIT_OPT)) {
         // the SPLIT auto variant (10) for identity class maps: no class-map
         // load in the walk (list modes; ptxas spills the count-mode forms)
+        // EVENTS (dense outputs) on the auto variant: inline emission
+        if constexpr (MODE == MODE_EMIT_OPT) {
+            if (variant == 10 && so.chain_events)
+                return launch_staged_v<E, TIER, MODE, 32, 1, 32, 1, 1, 1, false, true>(tmap, mtext, st, g, so,
+                                                                                     smem_stt, s);
+        }
         if (variant == 10 && st.cmap_ident && st.stride == kIdentStride)
             return launch_staged_v<E, TIER, MODE, 32, 1, 32, 1, 1, 1, true>(tmap, mtext, st, g, so, smem_stt, s);
     }
