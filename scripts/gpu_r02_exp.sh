@@ -1,8 +1,11 @@
 #!/bin/bash
-# scratch recipe: SPLIT EVENTS with inline emission (DENSE instantiation)
-O=gpurun_out/exp23
+# evidence: ncu --set full of the EVENTS single pass (scan + gather) on C5 English 5K, 256 MiB
+O=gpurun_out/events
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "dense or split or configs_scaled or shard or variants" > $O/pytest.log 2>&1; echo "rc=$?" >> $O/pytest.log
-timeout 900 python scripts/exp_tiers.py --workloads c5-english-20000-28,c5-english-50000-28 --tiers auto --list --exact-cap >> $O/tiers.jsonl 2>> $O/tiers.err
-timeout 600 python scripts/exp_tiers.py --workloads c3 --tiers auto --list >> $O/tiers.jsonl 2>> $O/tiers.err
+timeout 900 ncu --set full --clock-control none -k regex:"k_scan_staged|k_gather" -s 1 -c 2 \
+  -o $O/prof_ev python scripts/prof_target.py --config c5-english-5000-28 --reps 1 --mode list > $O/ncu_ev.out 2>&1
+ncu -i $O/prof_ev.ncu-rep --page raw --csv > $O/prof_ev.raw.csv 2>/dev/null
+rm -f $O/prof_ev.ncu-rep
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_ev.csv \
+  python scripts/prof_target.py --config c5-english-5000-28 --reps 2 --mode list > $O/ncu_l.out 2>&1
